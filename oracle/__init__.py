@@ -1,0 +1,132 @@
+"""CPU oracle for the NAS BT/SP ``compute_rhs`` pass -- TEST INFRASTRUCTURE ONLY.
+
+Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s ``cpu_baseline``
+/ ``--impl reference`` legs may import this package.  It wraps the plain C
+transcription in ``nas_oracle.c`` (NPB 3.x rhs.f as recalled in SURVEY.md
+App. A; the paper names NPB BT/SP at PAPER.md L1330-1362, L1470-1488 but never
+writes the loop nest) and shares no code with ``paper_conf_icpp_tiankexc16_b200``.
+
+Arrays cross this wrapper in the *logical* layout ``(nz, ny, nx, 5)`` float64
+(C order, component fastest), the layout ``nasgen`` produces; the wrapper pads
+to the NAS-BT layout ``u[nz][ny'][nx'][5]`` the C code uses.
+
+Pins: see ``tests/test_oracle_pins.py`` (P1-P6).  The NAS
+constants vs the NPB source are "parity unpinned" (reading c2).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+import threading
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SRC = os.path.join(_HERE, "nas_oracle.c")
+_HDR = os.path.join(_HERE, "nas_oracle.h")
+_LIB = os.path.join(_HERE, "libnas_oracle.so")
+
+# Strict IEEE: no FMA contraction, no reassociation (reading c6).
+CFLAGS = ["-O2", "-std=c99", "-fPIC", "-shared", "-fopenmp",
+          "-ffp-contract=off", "-fno-fast-math", "-fno-unsafe-math-optimizations"]
+
+_FIELDS = (
+    "dt c1 c2 c3 c4 c5 c1c2 c1c5 c3c4 conz1 con43 con16 dnxm1 dnym1 dnzm1 "
+    "tx1 tx2 tx3 ty1 ty2 ty3 tz1 tz2 tz3 dx1 dx2 dx3 dx4 dx5 dy1 dy2 dy3 dy4 dy5 "
+    "dz1 dz2 dz3 dz4 dz5 dssp dx1tx1 dx2tx1 dx3tx1 dx4tx1 dx5tx1 "
+    "dy1ty1 dy2ty1 dy3ty1 dy4ty1 dy5ty1 dz1tz1 dz2tz1 dz3tz1 dz4tz1 dz5tz1 "
+    "c3c4tx3 c3c4ty3 c3c4tz3 xxcon1 xxcon2 xxcon3 xxcon4 xxcon5 "
+    "yycon1 yycon2 yycon3 yycon4 yycon5 zzcon1 zzcon2 zzcon3 zzcon4 zzcon5"
+).split()
+
+
+class OracleConsts(ctypes.Structure):
+    _fields_ = [(f, ctypes.c_double) for f in _FIELDS]
+
+    def as_dict(self) -> dict:
+        return {f: getattr(self, f) for f in _FIELDS}
+
+
+_lock = threading.Lock()
+_lib = None
+
+
+def build(force: bool = False) -> str:
+    """Compile the oracle shared library in-tree with gcc (idempotent)."""
+    stale = (not os.path.exists(_LIB) or
+             os.path.getmtime(_LIB) < max(os.path.getmtime(_SRC), os.path.getmtime(_HDR)))
+    if force or stale:
+        tmp = _LIB + f".tmp{os.getpid()}"
+        subprocess.check_call(["gcc", *CFLAGS, "-o", tmp, _SRC])
+        os.replace(tmp, _LIB)
+    return _LIB
+
+
+def _load():
+    global _lib
+    with _lock:
+        if _lib is None:
+            lib = ctypes.CDLL(build())
+            lib.oracle_set_constants.argtypes = [ctypes.c_int] * 3 + [
+                ctypes.c_double, ctypes.POINTER(OracleConsts)]
+            lib.oracle_set_constants.restype = ctypes.c_int
+            lib.oracle_padded.argtypes = [ctypes.c_int]
+            lib.oracle_padded.restype = ctypes.c_int
+            dp = ctypes.POINTER(ctypes.c_double)
+            lib.oracle_compute_rhs.argtypes = [ctypes.c_int] * 3 + [
+                ctypes.POINTER(OracleConsts), dp, dp, dp, ctypes.c_int]
+            lib.oracle_compute_rhs.restype = ctypes.c_int
+            _lib = lib
+    return _lib
+
+
+def set_constants(nx: int, ny: int, nz: int, dt: float) -> OracleConsts:
+    """NPB set_constants as computed by the C oracle."""
+    c = OracleConsts()
+    if _load().oracle_set_constants(nx, ny, nz, dt, ctypes.byref(c)) != 0:
+        raise ValueError("oracle_set_constants: bad extents")
+    return c
+
+
+def padded(n: int) -> int:
+    return _load().oracle_padded(n)
+
+
+def to_nas(a: np.ndarray) -> np.ndarray:
+    """(nz, ny, nx, 5) -> zero-padded NAS-BT layout (nz, ny', nx', 5)."""
+    nz, ny, nx, _ = a.shape
+    out = np.zeros((nz, padded(ny), padded(nx), 5), dtype=np.float64)
+    out[:, :ny, :nx, :] = a
+    return out
+
+
+def from_nas(a: np.ndarray, nx: int, ny: int) -> np.ndarray:
+    return np.ascontiguousarray(a[:, :ny, :nx, :])
+
+
+def compute_rhs(u: np.ndarray, forcing: np.ndarray, dt: float | None = None,
+                consts: OracleConsts | None = None, threads: int = 1) -> np.ndarray:
+    """One NAS compute_rhs pass on the CPU.
+
+    ``u`` and ``forcing`` have logical shape (nz, ny, nx, 5) float64.  Either
+    ``dt`` (constants from NAS set_constants) or an explicit ``consts`` must be
+    given.  Returns rhs with the same logical shape.
+    """
+    if u.shape != forcing.shape or u.ndim != 4 or u.shape[3] != 5:
+        raise ValueError("u / forcing must both have shape (nz, ny, nx, 5)")
+    nz, ny, nx, _ = u.shape
+    if consts is None:
+        if dt is None:
+            raise ValueError("give dt or consts")
+        consts = set_constants(nx, ny, nz, dt)
+    un = to_nas(np.asarray(u, dtype=np.float64))
+    fn = to_nas(np.asarray(forcing, dtype=np.float64))
+    rn = np.zeros_like(un)
+    dp = ctypes.POINTER(ctypes.c_double)
+    rc = _load().oracle_compute_rhs(nx, ny, nz, ctypes.byref(consts),
+                                    un.ctypes.data_as(dp), fn.ctypes.data_as(dp),
+                                    rn.ctypes.data_as(dp), int(threads))
+    if rc != 0:
+        raise ValueError(f"oracle_compute_rhs failed ({rc}): extents must be >= 6")
+    return from_nas(rn, nx, ny)
