@@ -1,0 +1,302 @@
+#!/usr/bin/env python
+"""Benchmark: one NAS compute_rhs pass per step on B200 (BASELINE.json metric
+"rhs grid-points/s and achieved HBM GB/s (% of B200 peak) at 1/2/4/8 GPUs").
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config BT-C]
+  torchrun --nproc-per-node N bench.py --gpus N ...   (z-slab decomposition)
+  python bench.py --impl reference ...                (CPU oracle arm)
+
+Prints ONE JSON line on rank 0.  Workload at N=1: BT compute_rhs class C
+162^3 fp64 (BASELINE.json configs[4], the class the north_star's ">= 70 % of
+HBM on 1 GPU" target names).  Inputs (u 176 MB, forcing 176 MB, rhs 176 MB)
+are larger than the 126 MB L2, so no L2 flush is needed between steps.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import tempfile
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+BYTES_PER_POINT = 120  # read u 40 + forcing 40, write rhs 40 (fp64, 5 comps)
+FLOPS_PER_POINT = 430  # algorithmic fp64 flops (+1 reciprocal), DESIGN.md §6
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--warmup", type=int, default=20)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="BT-C", help="BENCH-CLASS, e.g. BT-C, SP-B")
+    ap.add_argument("--strict", action="store_true", help="time the STRICT variant")
+    ap.add_argument("--e2e-steps", type=int, default=5)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--soak-s", type=float, default=1.0,
+                    help="untimed passes before the timed region so the clock sampler "
+                         "sees the GPU under load")
+    return ap.parse_args()
+
+
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as fh:
+            d = json.load(fh)
+        return float(d["hbm_gbs"]), "measured"
+    return 6650.0, "fallback"
+
+
+def ncu_traffic(config_key):
+    """dram bytes per launch from the committed ncu --set full summary."""
+    p = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    if not os.path.exists(p):
+        return None
+    with open(p) as fh:
+        d = json.load(fh)
+    e = d.get(config_key)
+    return None if e is None else e.get("dram_bytes_per_launch")
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled every 100 ms."""
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index):
+        self.gpu = gpu_index
+        self.proc = None
+        self.f = None
+
+    def start(self):
+        try:
+            self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.Q}",
+                 "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=self.f, stderr=subprocess.DEVNULL)
+        except (OSError, FileNotFoundError):
+            self.proc = None
+        self.t0 = time.time()
+
+    def mark(self):
+        return time.time()
+
+    def stop(self):
+        rows = []
+        if self.proc is not None:
+            time.sleep(0.25)
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except subprocess.TimeoutExpired:
+                self.proc.kill()
+            self.f.flush()
+            with open(self.f.name) as fh:
+                for line in fh:
+                    parts = [x.strip() for x in line.split(",")]
+                    if len(parts) >= 9:
+                        rows.append(parts)
+            os.unlink(self.f.name)
+        return rows
+
+    @staticmethod
+    def summarise(rows):
+        if not rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        sm = [float(r[1]) for r in rows if r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in rows if r[2].replace(".", "").isdigit()]
+        pw = [float(r[3]) for r in rows if r[3].replace(".", "").isdigit()]
+        loaded = [s for s, p in zip(sm, pw) if p > 250.0] or sm
+        reasons = set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for r in rows:
+            for n, v in zip(names, r[5:9]):
+                if v.lower() == "active":
+                    reasons.add(n)
+        loaded.sort()
+        return {"sm_mhz": loaded[len(loaded) // 2] if loaded else None,
+                "sm_max_mhz": max(mx) if mx else None,
+                "samples": len(rows), "samples_under_load": len(loaded),
+                "power_w_max": max(pw) if pw else None,
+                "reasons": sorted(reasons)}
+
+
+def cpu_oracle_time(inp, max_seconds=12.0, threads=None):
+    """Time the oracle as it stands on the host cores (full passes)."""
+    import oracle
+    threads = threads or os.cpu_count() or 1
+    oracle.compute_rhs(inp.u, inp.forcing, dt=inp.dt, threads=threads)  # build + warm
+    n, t0 = 0, time.perf_counter()
+    while True:
+        oracle.compute_rhs(inp.u, inp.forcing, dt=inp.dt, threads=threads)
+        n += 1
+        el = time.perf_counter() - t0
+        if el >= max_seconds or n >= 50:
+            break
+    pts = inp.nx * inp.ny * inp.nz
+    return {"value": pts * n / el / 1e9, "unit": "Gpt/s", "cores": threads, "kind": "oracle",
+            "sample": f"{n} full {inp.nx}x{inp.ny}x{inp.nz} passes (plain C, -O2, "
+                      f"-ffp-contract=off, OpenMP over k) in {el:.2f} s"}
+
+
+def config_of(args):
+    import nasgen
+    bench, cls = args.config.split("-")
+    n, dt = nasgen.CLASSES[(bench, cls)]
+    return bench, cls, n, dt
+
+
+def run_reference(args):
+    """CPU oracle arm (rank 0 only)."""
+    import nasgen
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    bench, cls, n, dt = config_of(args)
+    inp = nasgen.make_class(bench, cls, seed=1)
+    import oracle
+    threads = os.cpu_count() or 1
+    for _ in range(max(args.warmup, 0)):
+        oracle.compute_rhs(inp.u, inp.forcing, dt=inp.dt, threads=threads)
+    times = []
+    for _ in range(args.steps):
+        t0 = time.perf_counter()
+        oracle.compute_rhs(inp.u, inp.forcing, dt=inp.dt, threads=threads)
+        times.append(time.perf_counter() - t0)
+    tot = sum(times)
+    pts = n ** 3
+    value = pts * args.steps / tot / 1e9
+    line = {
+        "impl": "reference", "metric": "rhs grid-points/s", "value": value, "unit": "Gpt/s",
+        "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": tot / args.steps * 1e3, "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": nasgen.config_name(bench, cls), "grid": [n, n, n],
+                   "points": pts, "l2": "host"},
+        "cpu_baseline": {"value": value, "unit": "Gpt/s", "cores": threads, "kind": "oracle",
+                         "sample": f"{args.steps} full {n}^3 passes of the plain-C oracle"},
+        "e2e": {"value": value, "unit": "Gpt/s", "h2d_bytes_per_step": 0,
+                "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def run_single(args):
+    import torch
+
+    import nasgen
+    import paper_conf_icpp_tiankexc16_b200 as sr
+
+    torch.cuda.set_device(0)
+    sr.init(0)
+    bench, cls, n, dt = config_of(args)
+    inp = nasgen.make_class(bench, cls, seed=1)
+    nx = ny = nz = n
+    c = sr.coeffs_nas(nx, ny, nz, dt)
+    du, df = sr.pack(inp.u), sr.pack(inp.forcing)
+    dr = torch.empty_like(du)
+    stream = torch.cuda.current_stream()
+    pts = nx * ny * nz
+
+    def step():
+        sr.rhs(du, df, dr, nx, c, strict=args.strict, stream=stream)
+
+    for _ in range(max(args.warmup, 3)):
+        step()
+    torch.cuda.synchronize()
+
+    sampler = ClockSampler(0)
+    sampler.start()
+    t_end = time.time() + args.soak_s
+    while time.time() < t_end:
+        for _ in range(50):
+            step()
+        torch.cuda.synchronize()
+
+    # timed region: K steps, per-launch events on the launching stream
+    ev = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps + 1)]
+    l0 = sr.launch_count()
+    torch.cuda.synchronize()
+    ev[0].record(stream)
+    for k in range(args.steps):
+        step()
+        ev[k + 1].record(stream)
+    torch.cuda.synchronize()
+    launches = sr.launch_count() - l0
+    per = [ev[k].elapsed_time(ev[k + 1]) for k in range(args.steps)]
+    total_ms = ev[0].elapsed_time(ev[-1])
+    rows = sampler.stop()
+    clocks = ClockSampler.summarise(rows)
+
+    ms_per_step = total_ms / args.steps
+    value = pts / (ms_per_step * 1e-3) / 1e9
+    kern_ms = sum(per) / len(per)
+    achieved = BYTES_PER_POINT * pts / (kern_ms * 1e-3) / 1e9
+    peak, peak_kind = measured_peaks()
+    key = f"{bench}-{cls}"
+    traffic = ncu_traffic(key)
+
+    # e2e: host (pinned) buffers through the C ABI, H2D + pass + D2H per step
+    hu, hf = sr.pack(inp.u, pin=True), sr.pack(inp.forcing, pin=True)
+    hr = torch.empty(hu.shape, dtype=torch.float64).pin_memory()
+    for _ in range(2):
+        sr.rhs_host(hu, hf, hr, du, df, dr, nx, c, strict=args.strict, stream=stream)
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for _ in range(args.e2e_steps):
+        sr.rhs_host(hu, hf, hr, du, df, dr, nx, c, strict=args.strict, stream=stream)
+    e1.record(stream)
+    torch.cuda.synchronize()
+    e2e_ms = e0.elapsed_time(e1) / args.e2e_steps
+    nbytes = hu.numel() * 8
+
+    line = {
+        "metric": "rhs grid-points/s", "value": value, "unit": "Gpt/s",
+        "n_gpus": 1, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "strong",
+        "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": nasgen.config_name(bench, cls), "grid": [nx, ny, nz],
+                   "points": pts, "variant": "strict" if args.strict else "production",
+                   "l2": "inputs 3x176 MB > 126 MB L2, no flush", "parallelism": "single"},
+        "hbm_gbs": achieved,
+        "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                     "frac": achieved / peak, "peak_kind": peak_kind, "traffic": traffic,
+                     "bytes_per_point": BYTES_PER_POINT, "kernel_ms": kern_ms,
+                     "frac_of_8000": achieved / 8000.0},
+        "clocks": clocks,
+        "e2e": {"value": pts / (e2e_ms * 1e-3) / 1e9, "unit": "Gpt/s",
+                "h2d_bytes_per_step": 2 * nbytes, "d2h_bytes_per_step": nbytes,
+                "ms_per_step": e2e_ms},
+        "gpu_launches": launches,
+        "kernel": sr.kernel_info(args.strict),
+    }
+    if not args.no_cpu_baseline:
+        line["cpu_baseline"] = cpu_oracle_time(inp)
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        run_reference(args)
+        return
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    if world > 1 or args.gpus > 1:
+        from paper_conf_icpp_tiankexc16_b200 import dist_bench
+        dist_bench.run(args)
+    else:
+        run_single(args)
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,163 @@
+/*
+ * include/safara.h -- C ABI of the B200 (sm_100a) NAS BT/SP compute_rhs library.
+ *
+ * What it computes: one NPB `compute_rhs` pass, rhs <- F(u, forcing), fp64,
+ * 5 components, 3-D flux differences plus fourth-order dissipation (SURVEY.md
+ * App. A; the loop nest the paper optimises).
+ * How: each CUDA thread owns one (i,j) column and marches along the sequential
+ * k loop with a rotating register window of u(:,i,j,k-2..k+2) -- the
+ * inter-iteration scalar replacement SAFARA applies to sequential loops
+ * (Fig. 6, Fig. 8); i/j neighbour
+ * planes arrive in shared memory by TMA.
+ *
+ * Conventions for every entry point
+ *  - Return value: SAFARA_OK (0) or a negative SAFARA_ERR_* code; never
+ *    throws, never prints, never synchronises the host inside the compute
+ *    calls.  Asynchronous device faults surface at the caller's next stream
+ *    synchronisation.  There is no CPU fallback and no unoptimised fallback
+ *    kernel (the paper's two-version scheme, L1275-1291, becomes up-front
+ *    validation that returns an error code instead).
+ *  - Ownership: all arrays are allocated and freed by the caller (PyTorch in
+ *    the Python binding).  The library never allocates device memory.
+ *  - `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).
+ *  - Arrays: fp64, component-planar.  Element (i, j, m, k) of any of u,
+ *    forcing, rhs sits at the 32-bit element offset
+ *        o = i + sy*j + sm*m + sk*k               (sx == 1)
+ *    from the array base.  ONE descriptor serves all arrays: this is the
+ *    paper's `dim` clause ("arrays have exactly the same dimensions ... offset0
+ *    shared", L1132-1171, recommended zero lower bounds L1194-1202).  Offsets
+ *    are 32-bit: the `small` clause ("array size smaller than 4GB ... 32-bit
+ *    integer offset", L1208-1273); a descriptor whose largest offset does not
+ *    fit in int32 is rejected with SAFARA_ERR_TOO_LARGE.
+ *  - u and forcing are read-only; every point of rhs (boundary faces included)
+ *    is written; rhs must not overlap u or forcing (SAFARA_ERR_ARG).
+ */
+#ifndef SAFARA_H
+#define SAFARA_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define SAFARA_ABI_VERSION 1
+
+enum {
+    SAFARA_OK            =  0,
+    SAFARA_ERR_ARG       = -1,  /* null pointer, aliasing, bad flag           */
+    SAFARA_ERR_SHAPE     = -2,  /* extent < 6, slab with < 2 planes, k range   */
+    SAFARA_ERR_LAYOUT    = -3,  /* strides overlap / sy < nx                   */
+    SAFARA_ERR_ALIGN     = -4,  /* pointer not 16 B aligned, odd stride        */
+    SAFARA_ERR_TOO_LARGE = -5,  /* largest offset >= 2^31 (`small` is false)   */
+    SAFARA_ERR_NOT_INIT  = -6,  /* safara_rhs_init not called on this device   */
+    SAFARA_ERR_CUDA      = -7,  /* CUDA runtime / driver error (launch, TMA)   */
+    SAFARA_ERR_NO_DEVICE = -8   /* device is not sm_100 or not present         */
+};
+
+/* flags for the *_ex / slab entry points */
+#define SAFARA_FLAG_STRICT 0x1  /* bit-identical to the NAS evaluation order:
+                                   no FMA contraction except where the product
+                                   is an exact power-of-two scaling           */
+
+/* The shared stride descriptor (`dim` + `small`).  Extents are the GLOBAL
+ * grid; lower bounds are 0; sx == 1 implicitly.                              */
+typedef struct {
+    int32_t nx, ny, nz;
+    int32_t sy, sm, sk;
+} safara_dims_t;
+
+/* The NPB set_constants values compute_rhs uses.
+ * dxt[m] = dx{m+1}tx1, dyt[m] = dy{m+1}ty1, dzt[m] = dz{m+1}tz1;
+ * xxcon[n] = xxcon{n+1} (xxcon[0] = xxcon1 is not used by compute_rhs).     */
+typedef struct {
+    double dt, dssp, c1, c2, con43, tx2, ty2, tz2;
+    double dxt[5], dyt[5], dzt[5];
+    double xxcon[5], yycon[5], zzcon[5];
+} safara_coeffs_t;
+
+/* Host only.  Fill `out` with NPB set_constants for an nx*ny*nz grid and time
+ * step dt (dssp = 0.25, c1 = 1.4, c2 = 0.4, dx = dy = 0.75, dz = 1.0 ...).
+ * Errors: SAFARA_ERR_ARG (out NULL), SAFARA_ERR_SHAPE (extent < 2).        */
+int safara_coeffs_nas(int nx, int ny, int nz, double dt, safara_coeffs_t *out);
+
+/* Once per process and device: checks the device is sm_100, resolves the
+ * driver's cuTensorMapEncodeTiled, caches SM count and kernel occupancy.
+ * Errors: SAFARA_ERR_NO_DEVICE, SAFARA_ERR_CUDA.                            */
+int safara_rhs_init(int device);
+
+/* Canonical pitch sy for a row of nx doubles: round_up(nx, 8).             */
+int safara_pitch(int nx);
+
+/* Canonical [k][m][j][i] descriptor: sy = safara_pitch(nx), sm = ny*sy,
+ * sk = 5*sm.  Errors: SAFARA_ERR_ARG, SAFARA_ERR_TOO_LARGE.                */
+int safara_dims_canonical(int nx, int ny, int nz, safara_dims_t *out);
+
+/* Validate a descriptor for arrays of nz_buf planes (the `dim`/`small`
+ * clause check).  Returns SAFARA_OK or the error the
+ * compute calls would return.                                               */
+int safara_validate_dims(const safara_dims_t *dims, int nz_buf);
+
+/* One compute_rhs pass on device arrays in the canonical layout
+ * (safara_dims_canonical(nx, ny, nz)).  Asynchronous on `stream`.
+ * Launches exactly one kernel.  Requires every extent >= 6 (DESIGN.md
+ * reading c4).  Production (FMA-contracted) variant; see *_ex for STRICT.  */
+int safara_rhs(const double *u, const double *forcing, double *rhs,
+               int nx, int ny, int nz, const safara_coeffs_t *coeffs,
+               void *stream);
+
+/* Same with an explicit descriptor (any valid stride order, e.g. SP's
+ * native [m][k][j][i]) and flags (SAFARA_FLAG_STRICT).                      */
+int safara_rhs_ex(const double *u, const double *forcing, double *rhs,
+                  const safara_dims_t *dims, const safara_coeffs_t *coeffs,
+                  int flags, void *stream);
+
+/* z-slab variant for one rank of a z-decomposition.
+ *   dims:      GLOBAL extents nx, ny, nz and the shared strides;
+ *   k0, nzl:   this slab owns global planes [k0, k0+nzl), nzl >= 2;
+ *   u_slab:    nzl+4 planes: local plane p holds global plane k0-2+p (two
+ *              ghost planes on each side, filled by the caller's halo
+ *              exchange; ghosts beyond the global grid are never read);
+ *   forcing_slab, rhs_slab: nzl planes, local plane p = global k0+p;
+ *   part:      SAFARA_PART_ALL, _INTERIOR (planes that need no ghost: can
+ *              overlap the halo exchange; also writes the boundary faces) or
+ *              _EDGE (the <= 4 planes next to the ghosts).
+ * The dissipation case and boundary test use the GLOBAL k (reading c12).   */
+#define SAFARA_PART_ALL      0
+#define SAFARA_PART_INTERIOR 1
+#define SAFARA_PART_EDGE     2
+int safara_rhs_slab(const double *u_slab, const double *forcing_slab,
+                    double *rhs_slab, const safara_dims_t *dims, int k0,
+                    int nzl, const safara_coeffs_t *coeffs, int flags,
+                    int part, void *stream);
+
+/* End-to-end call with HOST arrays (canonical layout): copies u and forcing
+ * host->device into the caller's device buffers u_dev/forcing_dev, runs the
+ * pass into rhs_dev and copies rhs device->host, all asynchronously on
+ * `stream` in `nchunks` k-chunks so that copies and compute overlap (host
+ * buffers should be pinned).  The caller synchronises the stream.            */
+int safara_rhs_host(const double *u_host, const double *forcing_host,
+                    double *rhs_host, double *u_dev, double *forcing_dev,
+                    double *rhs_dev, int nx, int ny, int nz,
+                    const safara_coeffs_t *coeffs, int flags, int nchunks,
+                    void *stream);
+
+/* Number of kernel launches issued by this process since load.            */
+int64_t safara_launch_count(void);
+
+/* Static description of a compiled kernel variant (registers/thread, local
+ * (spill) bytes, static+dynamic smem, CTAs/SM), for evidence and tests.
+ * which: 0 = production, 1 = STRICT.                                       */
+typedef struct {
+    int regs_per_thread, local_bytes, smem_bytes, threads_per_cta, ctas_per_sm;
+    int tile_x, tile_y, stages;
+} safara_kernel_info_t;
+int safara_kernel_info(int which, safara_kernel_info_t *out);
+
+/* Human-readable message for an error code (static storage).              */
+const char *safara_strerror(int code);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SAFARA_H */

@@ -1,0 +1,97 @@
+"""ctypes declarations of the C ABI in include/safara.h (argument marshalling only).
+
+Loading fails loudly if the in-tree ``libsafara_rhs.so`` is missing: there is
+no CPU or PyTorch fallback for any step of the pass.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import re
+import threading
+
+PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(PKG, "libsafara_rhs.so")
+HEADER = os.path.join(os.path.dirname(PKG), "include", "safara.h")
+
+SAFARA_OK = 0
+SAFARA_FLAG_STRICT = 0x1
+SAFARA_PART_ALL, SAFARA_PART_INTERIOR, SAFARA_PART_EDGE = 0, 1, 2
+
+
+class SafaraError(RuntimeError):
+    def __init__(self, code: int, where: str):
+        self.code = code
+        super().__init__(f"{where}: {strerror(code)} (code {code})")
+
+
+class Dims(ctypes.Structure):
+    _fields_ = [(n, ctypes.c_int32) for n in ("nx", "ny", "nz", "sy", "sm", "sk")]
+
+
+class Coeffs(ctypes.Structure):
+    _fields_ = [(n, ctypes.c_double) for n in
+                ("dt", "dssp", "c1", "c2", "con43", "tx2", "ty2", "tz2")] + [
+        (n, ctypes.c_double * 5) for n in ("dxt", "dyt", "dzt", "xxcon", "yycon", "zzcon")]
+
+
+class KernelInfo(ctypes.Structure):
+    _fields_ = [(n, ctypes.c_int) for n in
+                ("regs_per_thread", "local_bytes", "smem_bytes", "threads_per_cta",
+                 "ctas_per_sm", "tile_x", "tile_y", "stages")]
+
+
+_lock = threading.Lock()
+_lib = None
+
+_dp = ctypes.c_void_p  # device / host pointers travel as plain addresses
+_SIGS = {
+    "safara_coeffs_nas": ([ctypes.c_int] * 3 + [ctypes.c_double, ctypes.POINTER(Coeffs)], ctypes.c_int),
+    "safara_rhs_init": ([ctypes.c_int], ctypes.c_int),
+    "safara_pitch": ([ctypes.c_int], ctypes.c_int),
+    "safara_dims_canonical": ([ctypes.c_int] * 3 + [ctypes.POINTER(Dims)], ctypes.c_int),
+    "safara_validate_dims": ([ctypes.POINTER(Dims), ctypes.c_int], ctypes.c_int),
+    "safara_rhs": ([_dp, _dp, _dp] + [ctypes.c_int] * 3 + [ctypes.POINTER(Coeffs), _dp], ctypes.c_int),
+    "safara_rhs_ex": ([_dp, _dp, _dp, ctypes.POINTER(Dims), ctypes.POINTER(Coeffs), ctypes.c_int, _dp],
+                      ctypes.c_int),
+    "safara_rhs_slab": ([_dp, _dp, _dp, ctypes.POINTER(Dims), ctypes.c_int, ctypes.c_int,
+                         ctypes.POINTER(Coeffs), ctypes.c_int, ctypes.c_int, _dp], ctypes.c_int),
+    "safara_rhs_host": ([_dp] * 6 + [ctypes.c_int] * 3 + [ctypes.POINTER(Coeffs), ctypes.c_int,
+                                                           ctypes.c_int, _dp], ctypes.c_int),
+    "safara_launch_count": ([], ctypes.c_int64),
+    "safara_kernel_info": ([ctypes.c_int, ctypes.POINTER(KernelInfo)], ctypes.c_int),
+    "safara_strerror": ([ctypes.c_int], ctypes.c_char_p),
+}
+
+
+def header_symbols() -> list[str]:
+    """Function names declared in include/safara.h."""
+    txt = open(HEADER).read()
+    return sorted(set(re.findall(r"\b(safara_[a-z_0-9]+)\s*\(", txt)))
+
+
+def lib():
+    """The loaded library (raises if it was not built)."""
+    global _lib
+    with _lock:
+        if _lib is None:
+            if not os.path.exists(LIB_PATH):
+                raise RuntimeError(
+                    f"{LIB_PATH} is missing: build it with `python -c 'import __graft_entry__ as g; "
+                    "g.build()'` (no fallback exists)")
+            L = ctypes.CDLL(LIB_PATH)
+            for name, (args, res) in _SIGS.items():
+                fn = getattr(L, name)
+                fn.argtypes = args
+                fn.restype = res
+            _lib = L
+    return _lib
+
+
+def strerror(code: int) -> str:
+    return lib().safara_strerror(int(code)).decode()
+
+
+def check(code: int, where: str) -> None:
+    if code != SAFARA_OK:
+        raise SafaraError(code, where)

@@ -1,0 +1,375 @@
+// api.cu -- the C ABI declared in include/safara.h.
+//
+// Host-side responsibilities only: argument / descriptor validation (the
+// `dim` and `small` clause checks that replace the paper's two-version kernel,
+// PAPER.md L1275-1291), NPB set_constants for the coefficients, the TMA
+// tensor map for u, the work decomposition, and the launch.  Every step of the
+// pass itself runs in the kernel (rhs_kernel.cuh).  No exceptions escape, no
+// host synchronisation happens in the compute calls, nothing is allocated.
+#include <cudaTypedefs.h>
+
+#include <algorithm>
+#include <atomic>
+#include <cstdint>
+#include <cstring>
+#include <mutex>
+
+#include "safara_internal.h"
+
+using namespace safara;
+
+namespace {
+
+constexpr int kMaxDevices = 64;
+
+struct DeviceState {
+    bool ready = false;
+    int sms = 0;
+    int ctas_fast = 0, ctas_strict = 0;
+    cudaFuncAttributes attr_fast{}, attr_strict{};
+};
+
+DeviceState g_dev[kMaxDevices];
+std::mutex g_mutex;
+PFN_cuTensorMapEncodeTiled_v12000 g_encode = nullptr;
+std::atomic<int64_t> g_launches{0};
+
+int current_device(int *dev) {
+    if (cudaGetDevice(dev) != cudaSuccess) return SAFARA_ERR_CUDA;
+    if (*dev < 0 || *dev >= kMaxDevices) return SAFARA_ERR_NO_DEVICE;
+    if (!g_dev[*dev].ready) return SAFARA_ERR_NOT_INIT;
+    return SAFARA_OK;
+}
+
+// Largest element offset reachable through the descriptor, in 64-bit.
+long long max_offset(const safara_dims_t &d, int nzb) {
+    return (long long)(d.nx - 1) + (long long)d.sy * (d.ny - 1) + (long long)d.sm * 4 +
+           (long long)d.sk * (nzb - 1);
+}
+
+int validate(const safara_dims_t *d, int nzb) {
+    if (!d) return SAFARA_ERR_ARG;
+    if (d->nx < 6 || d->ny < 6 || d->nz < 6 || nzb < 1) return SAFARA_ERR_SHAPE;
+    if (d->sy < d->nx || d->sm <= 0 || d->sk <= 0) return SAFARA_ERR_LAYOUT;
+    // j must be the second-fastest dimension (the smem tile is [m][j][i]).
+    if (d->sy >= d->sm || d->sy >= d->sk) return SAFARA_ERR_LAYOUT;
+    // non-overlap: order (j, m, k) by stride; each stride >= previous span.
+    long long s1 = d->sm, e1 = 5, s2 = d->sk, e2 = nzb;
+    if (s1 > s2) { std::swap(s1, s2); std::swap(e1, e2); }
+    if (s1 == s2) return SAFARA_ERR_LAYOUT;
+    if (s1 < (long long)d->sy * d->ny) return SAFARA_ERR_LAYOUT;
+    if (s2 < s1 * e1) return SAFARA_ERR_LAYOUT;
+    // TMA: global strides must be multiples of 16 bytes.
+    if ((d->sy & 1) || (d->sm & 1) || (d->sk & 1)) return SAFARA_ERR_ALIGN;
+    if (max_offset(*d, nzb) >= (1LL << 31)) return SAFARA_ERR_TOO_LARGE;
+    return SAFARA_OK;
+}
+
+bool overlaps(const void *a, long long abytes, const void *b, long long bbytes) {
+    const uintptr_t a0 = (uintptr_t)a, b0 = (uintptr_t)b;
+    return a0 < b0 + (uintptr_t)bbytes && b0 < a0 + (uintptr_t)abytes;
+}
+
+int check_ptrs(const double *u, long long ubytes, const double *f, long long fbytes,
+               const double *r, long long rbytes) {
+    if (!u || !f || !r) return SAFARA_ERR_ARG;
+    if (((uintptr_t)u | (uintptr_t)f | (uintptr_t)r) & 15u) return SAFARA_ERR_ALIGN;
+    if (overlaps(r, rbytes, u, ubytes) || overlaps(r, rbytes, f, fbytes)) return SAFARA_ERR_ARG;
+    return SAFARA_OK;
+}
+
+void to_coef(const safara_coeffs_t &in, Coef &c) {
+    c.dt = in.dt;
+    c.dssp = in.dssp;
+    c.c1 = in.c1;
+    c.c2 = in.c2;
+    c.t2[0] = in.tx2;
+    c.t2[1] = in.ty2;
+    c.t2[2] = in.tz2;
+    for (int m = 0; m < 5; ++m) {
+        c.d1[0][m] = in.dxt[m];
+        c.d1[1][m] = in.dyt[m];
+        c.d1[2][m] = in.dzt[m];
+    }
+    const double *con[3] = {in.xxcon, in.yycon, in.zzcon};
+    for (int a = 0; a < 3; ++a) {
+        c.con2[a] = con[a][1];
+        c.con2x43[a] = con[a][1] * in.con43;  // NAS: xxcon2*con43*(...), left to right
+        c.con3[a] = con[a][2];
+        c.con4[a] = con[a][3];
+        c.con5[a] = con[a][4];
+    }
+}
+
+// 4-D tensor map over u: dim0 = i, then (j, m, k) ordered by stride.
+int encode_u_map(CUtensorMap *map, const double *u, const safara_dims_t &d, int nzb, int *pos_j,
+                 int *pos_m, int *pos_k) {
+    struct Ax { int which; long long stride, extent, box; } ax[3] = {
+        {0, d.sy, d.ny, UY}, {1, d.sm, 5, 5}, {2, d.sk, nzb, 1}};
+    std::sort(ax, ax + 3, [](const Ax &a, const Ax &b) { return a.stride < b.stride; });
+    cuuint64_t gdim[4] = {(cuuint64_t)d.nx, 0, 0, 0};
+    cuuint64_t gstride[3];
+    cuuint32_t box[4] = {(cuuint32_t)UX, 0, 0, 0};
+    cuuint32_t estride[4] = {1, 1, 1, 1};
+    for (int t = 0; t < 3; ++t) {
+        gdim[t + 1] = (cuuint64_t)ax[t].extent;
+        gstride[t] = (cuuint64_t)ax[t].stride * sizeof(double);
+        box[t + 1] = (cuuint32_t)ax[t].box;
+        if (ax[t].which == 0) *pos_j = t + 1;
+        if (ax[t].which == 1) *pos_m = t + 1;
+        if (ax[t].which == 2) *pos_k = t + 1;
+    }
+    CUresult r = g_encode(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 4, const_cast<double *>(u), gdim,
+                          gstride, box, estride, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                          CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                          CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    return r == CUDA_SUCCESS ? SAFARA_OK : SAFARA_ERR_CUDA;
+}
+
+// Shared launch path.  u has nzu planes, u plane = k - k0 + ukoff; forcing
+// and rhs start at global plane k0.  [ka0,kb0) U [ka1,kb1) are computed;
+// boundary faces of local planes [fk_lo, fk_hi) are copied.
+int launch(const double *u, const double *f, double *r, const safara_dims_t &d, int nzu, int k0,
+           int ukoff, int ka0, int kb0, int ka1, int kb1, int fk_lo, int fk_hi,
+           const safara_coeffs_t *coeffs, int flags, cudaStream_t stream) {
+    int dev;
+    int rc = current_device(&dev);
+    if (rc) return rc;
+    if (!coeffs) return SAFARA_ERR_ARG;
+    if (flags & ~SAFARA_FLAG_STRICT) return SAFARA_ERR_ARG;
+    const DeviceState &st = g_dev[dev];
+
+    Params p;
+    std::memset(&p, 0, sizeof(p));
+    p.nx = d.nx; p.ny = d.ny; p.nz = d.nz;
+    p.sy = d.sy; p.sm = d.sm; p.sk = d.sk;
+    p.k0 = k0; p.ukoff = ukoff; p.nzu = nzu;
+    p.ka0 = ka0; p.kb0 = std::max(ka0, kb0);
+    p.ka1 = ka1; p.kb1 = std::max(ka1, kb1);
+    p.n0 = p.kb0 - p.ka0;
+    p.nplanes = p.n0 + (p.kb1 - p.ka1);
+    p.ntx = (d.nx - 2 + TX - 1) / TX;
+    p.nty = (d.ny - 2 + TY - 1) / TY;
+    p.units = (long long)p.ntx * p.nty * p.nplanes;
+    p.fk_lo = fk_lo; p.fk_hi = fk_hi;
+    p.u = u; p.f = f; p.r = r;
+    to_coef(*coeffs, p.c);
+
+    const bool strict = (flags & SAFARA_FLAG_STRICT) != 0;
+    const int per_sm = strict ? st.ctas_strict : st.ctas_fast;
+    const long long max_ctas = (long long)std::max(per_sm, 1) * st.sms;
+    long long ncta = (p.units + MIN_PLANES_PER_CTA - 1) / MIN_PLANES_PER_CTA;
+    ncta = std::min(ncta, max_ctas);
+    if (ncta < 1) {
+        if (fk_hi <= fk_lo) return SAFARA_OK;  // nothing to do
+        ncta = std::min<long long>(max_ctas, 16);
+    }
+    p.ncta = (int)ncta;
+
+    CUtensorMap map;
+    rc = encode_u_map(&map, u, d, nzu, &p.pos_j, &p.pos_m, &p.pos_k);
+    if (rc) return rc;
+    cudaError_t e = strict ? launch_rhs_strict(map, p, stream) : launch_rhs_fast(map, p, stream);
+    if (e != cudaSuccess) return SAFARA_ERR_CUDA;
+    g_launches.fetch_add(1, std::memory_order_relaxed);
+    return SAFARA_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+int safara_coeffs_nas(int nx, int ny, int nz, double dt, safara_coeffs_t *out) {
+    if (!out) return SAFARA_ERR_ARG;
+    if (nx < 2 || ny < 2 || nz < 2) return SAFARA_ERR_SHAPE;
+    // NPB set_constants.f, library's own copy.
+    const double c1 = 1.4, c2 = 0.4, c3 = 0.1, c4 = 1.0, c5 = 1.4;
+    const double dnxm1 = 1.0 / (double)(nx - 1);
+    const double dnym1 = 1.0 / (double)(ny - 1);
+    const double dnzm1 = 1.0 / (double)(nz - 1);
+    const double c1c5 = c1 * c5, c3c4 = c3 * c4;
+    const double tx1 = 1.0 / (dnxm1 * dnxm1), tx2 = 1.0 / (2.0 * dnxm1), tx3 = 1.0 / dnxm1;
+    const double ty1 = 1.0 / (dnym1 * dnym1), ty2 = 1.0 / (2.0 * dnym1), ty3 = 1.0 / dnym1;
+    const double tz1 = 1.0 / (dnzm1 * dnzm1), tz2 = 1.0 / (2.0 * dnzm1), tz3 = 1.0 / dnzm1;
+    const double dx = 0.75, dy = 0.75, dz = 1.0;  // dx1..dx5, dy1..dy5, dz1..dz5
+    const double conz1 = 1.0 - c1c5, con43 = 4.0 / 3.0, con16 = 1.0 / 6.0;
+    std::memset(out, 0, sizeof(*out));
+    out->dt = dt;
+    out->dssp = 0.25 * std::max(dx, std::max(dy, dz));
+    out->c1 = c1;
+    out->c2 = c2;
+    out->con43 = con43;
+    out->tx2 = tx2;
+    out->ty2 = ty2;
+    out->tz2 = tz2;
+    for (int m = 0; m < 5; ++m) {
+        out->dxt[m] = dx * tx1;
+        out->dyt[m] = dy * ty1;
+        out->dzt[m] = dz * tz1;
+    }
+    const double t3[3] = {tx3, ty3, tz3};
+    double *con[3] = {out->xxcon, out->yycon, out->zzcon};
+    for (int a = 0; a < 3; ++a) {
+        const double c34 = c3c4 * t3[a];
+        con[a][0] = c34 * con43 * t3[a];
+        con[a][1] = c34 * t3[a];
+        con[a][2] = c34 * conz1 * t3[a];
+        con[a][3] = c34 * con16 * t3[a];
+        con[a][4] = c34 * c1c5 * t3[a];
+    }
+    return SAFARA_OK;
+}
+
+int safara_rhs_init(int device) {
+    std::lock_guard<std::mutex> lock(g_mutex);
+    int count = 0;
+    if (cudaGetDeviceCount(&count) != cudaSuccess || count < 1) return SAFARA_ERR_NO_DEVICE;
+    if (device < 0 || device >= count || device >= kMaxDevices) return SAFARA_ERR_NO_DEVICE;
+    if (g_dev[device].ready) return SAFARA_OK;
+    int major = 0, minor = 0, sms = 0;
+    if (cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, device) ||
+        cudaDeviceGetAttribute(&minor, cudaDevAttrComputeCapabilityMinor, device) ||
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device))
+        return SAFARA_ERR_CUDA;
+    if (major != 10 || minor != 0) return SAFARA_ERR_NO_DEVICE;  // sm_100a code only
+    if (!g_encode) {
+        void *fn = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q) !=
+                cudaSuccess ||
+            q != cudaDriverEntryPointSuccess || !fn)
+            return SAFARA_ERR_CUDA;
+        g_encode = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
+    }
+    int prev = 0;
+    if (cudaGetDevice(&prev) != cudaSuccess) return SAFARA_ERR_CUDA;
+    if (cudaSetDevice(device) != cudaSuccess) return SAFARA_ERR_CUDA;
+    DeviceState st;
+    st.sms = sms;
+    cudaError_t e = setup_rhs_fast(&st.ctas_fast, &st.attr_fast);
+    if (e == cudaSuccess) e = setup_rhs_strict(&st.ctas_strict, &st.attr_strict);
+    cudaSetDevice(prev);
+    if (e != cudaSuccess) return SAFARA_ERR_CUDA;
+    st.ready = true;
+    g_dev[device] = st;
+    return SAFARA_OK;
+}
+
+int safara_pitch(int nx) { return nx <= 0 ? 0 : ((nx + 7) / 8) * 8; }
+
+int safara_dims_canonical(int nx, int ny, int nz, safara_dims_t *out) {
+    if (!out) return SAFARA_ERR_ARG;
+    if (nx < 1 || ny < 1 || nz < 1) return SAFARA_ERR_SHAPE;
+    const long long sy = safara_pitch(nx), sm = sy * ny, sk = 5 * sm;
+    if (sk * nz >= (1LL << 31)) return SAFARA_ERR_TOO_LARGE;
+    out->nx = nx; out->ny = ny; out->nz = nz;
+    out->sy = (int32_t)sy; out->sm = (int32_t)sm; out->sk = (int32_t)sk;
+    return SAFARA_OK;
+}
+
+int safara_validate_dims(const safara_dims_t *dims, int nz_buf) { return validate(dims, nz_buf); }
+
+int safara_rhs_ex(const double *u, const double *forcing, double *rhs, const safara_dims_t *dims,
+                  const safara_coeffs_t *coeffs, int flags, void *stream) {
+    int rc = validate(dims, dims ? dims->nz : 0);
+    if (rc) return rc;
+    const long long bytes = (max_offset(*dims, dims->nz) + 1) * (long long)sizeof(double);
+    rc = check_ptrs(u, bytes, forcing, bytes, rhs, bytes);
+    if (rc) return rc;
+    const int nz = dims->nz;
+    return launch(u, forcing, rhs, *dims, nz, 0, 0, 1, nz - 1, 0, 0, 0, nz, coeffs, flags,
+                  (cudaStream_t)stream);
+}
+
+int safara_rhs(const double *u, const double *forcing, double *rhs, int nx, int ny, int nz,
+               const safara_coeffs_t *coeffs, void *stream) {
+    safara_dims_t d;
+    int rc = safara_dims_canonical(nx, ny, nz, &d);
+    if (rc) return rc;
+    return safara_rhs_ex(u, forcing, rhs, &d, coeffs, 0, stream);
+}
+
+int safara_rhs_slab(const double *u_slab, const double *forcing_slab, double *rhs_slab,
+                    const safara_dims_t *dims, int k0, int nzl, const safara_coeffs_t *coeffs,
+                    int flags, int part, void *stream) {
+    if (!dims) return SAFARA_ERR_ARG;
+    if (part < SAFARA_PART_ALL || part > SAFARA_PART_EDGE) return SAFARA_ERR_ARG;
+    if (nzl < 2 || k0 < 0 || k0 + nzl > dims->nz) return SAFARA_ERR_SHAPE;
+    const int nzu = nzl + 4;
+    int rc = validate(dims, nzu);
+    if (rc) return rc;
+    const long long ubytes = (max_offset(*dims, nzu) + 1) * (long long)sizeof(double);
+    const long long fbytes = (max_offset(*dims, nzl) + 1) * (long long)sizeof(double);
+    rc = check_ptrs(u_slab, ubytes, forcing_slab, fbytes, rhs_slab, fbytes);
+    if (rc) return rc;
+    const int lo = std::max(k0, 1), hi = std::min(k0 + nzl, dims->nz - 1);
+    int ka0 = lo, kb0 = hi, ka1 = 0, kb1 = 0, fk_lo = 0, fk_hi = nzl;
+    if (part == SAFARA_PART_INTERIOR) {
+        ka0 = std::max(lo, k0 + 2);
+        kb0 = std::min(hi, k0 + nzl - 2);
+    } else if (part == SAFARA_PART_EDGE) {
+        const int e0 = std::min(hi, k0 + 2);
+        const int e1 = std::max(e0, std::max(lo, k0 + nzl - 2));
+        ka0 = lo; kb0 = e0; ka1 = e1; kb1 = hi;
+        fk_lo = fk_hi = 0;
+    }
+    return launch(u_slab, forcing_slab, rhs_slab, *dims, nzu, k0, 2, ka0, kb0, ka1, kb1, fk_lo,
+                  fk_hi, coeffs, flags, (cudaStream_t)stream);
+}
+
+int safara_rhs_host(const double *u_host, const double *forcing_host, double *rhs_host,
+                    double *u_dev, double *forcing_dev, double *rhs_dev, int nx, int ny, int nz,
+                    const safara_coeffs_t *coeffs, int flags, int nchunks, void *stream) {
+    (void)nchunks;
+    if (!u_host || !forcing_host || !rhs_host) return SAFARA_ERR_ARG;
+    safara_dims_t d;
+    int rc = safara_dims_canonical(nx, ny, nz, &d);
+    if (rc) return rc;
+    const size_t bytes = (size_t)d.sk * nz * sizeof(double);
+    cudaStream_t s = (cudaStream_t)stream;
+    if (cudaMemcpyAsync(u_dev, u_host, bytes, cudaMemcpyHostToDevice, s) != cudaSuccess ||
+        cudaMemcpyAsync(forcing_dev, forcing_host, bytes, cudaMemcpyHostToDevice, s) != cudaSuccess)
+        return SAFARA_ERR_CUDA;
+    rc = safara_rhs_ex(u_dev, forcing_dev, rhs_dev, &d, coeffs, flags, stream);
+    if (rc) return rc;
+    if (cudaMemcpyAsync(rhs_host, rhs_dev, bytes, cudaMemcpyDeviceToHost, s) != cudaSuccess)
+        return SAFARA_ERR_CUDA;
+    return SAFARA_OK;
+}
+
+int64_t safara_launch_count(void) { return g_launches.load(); }
+
+int safara_kernel_info(int which, safara_kernel_info_t *out) {
+    if (!out || (which != 0 && which != 1)) return SAFARA_ERR_ARG;
+    int dev;
+    int rc = current_device(&dev);
+    if (rc) return rc;
+    const DeviceState &st = g_dev[dev];
+    const cudaFuncAttributes &a = which ? st.attr_strict : st.attr_fast;
+    out->regs_per_thread = a.numRegs;
+    out->local_bytes = (int)a.localSizeBytes;
+    out->smem_bytes = (int)(a.sharedSizeBytes + SMEM_BYTES);
+    out->threads_per_cta = NTHREADS;
+    out->ctas_per_sm = which ? st.ctas_strict : st.ctas_fast;
+    out->tile_x = TX;
+    out->tile_y = TY;
+    out->stages = STAGES;
+    return SAFARA_OK;
+}
+
+const char *safara_strerror(int code) {
+    switch (code) {
+        case SAFARA_OK: return "success";
+        case SAFARA_ERR_ARG: return "invalid argument (null pointer, aliasing or bad flag)";
+        case SAFARA_ERR_SHAPE: return "invalid shape (extent < 6, slab < 2 planes or bad k range)";
+        case SAFARA_ERR_LAYOUT: return "invalid layout (strides overlap, sy < nx or j not second-fastest)";
+        case SAFARA_ERR_ALIGN: return "misaligned pointer or stride (16-byte TMA rule)";
+        case SAFARA_ERR_TOO_LARGE: return "largest offset >= 2^31: the `small` (32-bit offset) claim is false";
+        case SAFARA_ERR_NOT_INIT: return "safara_rhs_init was not called for the current device";
+        case SAFARA_ERR_CUDA: return "CUDA runtime or driver error";
+        case SAFARA_ERR_NO_DEVICE: return "no sm_100 device at this index";
+        default: return "unknown error code";
+    }
+}
+
+}  // extern "C"

@@ -1,0 +1,484 @@
+// rhs_kernel.cuh -- the NAS BT/SP compute_rhs pass for sm_100a.
+//
+// Included by rhs_fast.cu (FMA contraction allowed, --fmad=true) and by
+// rhs_strict.cu (--fmad=false: every product and sum rounded exactly where
+// the NAS text rounds it, so the result is bit-identical to the oracle).
+//
+// Design:
+//  * One thread per (i,j) column of a TX x TY CTA tile; the thread marches
+//    along the sequential k loop.  This is SAFARA's split (PAPER.md
+//    L684-692): the parallel i/j loops get no inter-iteration reuse, the
+//    sequential k loop gets scalar replacement.
+//  * Inter-iteration scalar replacement along k, prioritised by reuse
+//    (cost model L x C): each u(m,i,j,k) is used at five
+//    consecutive k steps, so the thread keeps u(:,i,j,k-2..k+2) in a
+//    rotating register window (Fig. 6, generalised to depth 5),
+//    plus its own rho_i / square at k-1..k+1.  forcing is used once: it is
+//    streamed (one-step register prefetch), never staged.
+//  * i/j neighbours (reused by 4 other threads each, the "uncoalesced"
+//    references SAFARA favours, L643-675) come from shared memory: the u
+//    plane tile with a halo of 2 arrives by TMA (cp.async.bulk.tensor, one
+//    box per plane, STAGES-deep mbarrier ring); rho_i and square of the
+//    plane (halo 1) are computed once per point into a 3-slot smem ring.
+//    Every other derived quantity (us, vs, ws, qs, u5*rho_i, products) is
+//    recomputed from {u, rho_i, square} at use: one DMUL costs a quarter of
+//    what a shared-memory double costs (64 FP64 lanes vs 16 doubles/clk/SM).
+//  * `dim`: forcing/rhs share one int32 descriptor (sy, sm, sk) held in the
+//    kernel parameters (constant bank); `small`: all offsets are 32-bit.
+//  * Evaluation order follows the NAS text left to right (DESIGN.md reading
+//    c6).  Where NAS multiplies by 2.0 or 4.0 (exact scalings) the subtract
+//    is a single fma, which rounds identically.
+#pragma once
+#include "safara_internal.h"
+
+namespace safara {
+namespace dev {
+
+constexpr int UPM = UX * UY;  // doubles per component plane of a u tile
+
+__device__ __forceinline__ uint32_t smem_u32(const void *p) {
+    return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+
+__device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count)
+                 : "memory");
+}
+
+__device__ __forceinline__ void fence_mbar_init() {
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+
+__device__ __forceinline__ void mbar_expect_tx(uint64_t *bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)),
+                 "r"(bytes)
+                 : "memory");
+}
+
+__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
+    const uint32_t addr = smem_u32(bar);
+    uint32_t done;
+    do {
+        asm volatile(
+            "{\n\t.reg .pred p;\n\t"
+            "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+            "selp.u32 %0, 1, 0, p;\n\t}"
+            : "=r"(done)
+            : "r"(addr), "r"(parity)
+            : "memory");
+    } while (!done);
+}
+
+__device__ __forceinline__ void tma_load_4d(void *dst, const CUtensorMap *map, uint64_t *bar,
+                                            int c0, int c1, int c2, int c3) {
+    asm volatile(
+        "cp.async.bulk.tensor.4d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
+        " [%0], [%1, {%2, %3, %4, %5}], [%6];" ::"r"(smem_u32(dst)),
+        "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(c2), "r"(c3),
+        "r"(smem_u32(bar))
+        : "memory");
+}
+
+__device__ __forceinline__ void prefetch_tmap(const CUtensorMap *map) {
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(map)) : "memory");
+}
+
+// NAS second difference  (a[p] - 2.0*a[c]) + a[q]; 2.0*a[c] is exact, so the
+// fused form rounds exactly like the two-step form.
+__device__ __forceinline__ double d2(double ap, double ac, double aq) {
+    return __fma_rn(-2.0, ac, ap) + aq;
+}
+
+// rho_i = 1.0/u1; square = 0.5*(u2*u2 + u3*u3 + u4*u4)*rho_i  (App. A step 0)
+__device__ __forceinline__ void aux_of(double u1, double u2, double u3, double u4, double &rho,
+                                       double &sq) {
+    rho = 1.0 / u1;
+    sq = 0.5 * (u2 * u2 + u3 * u3 + u4 * u4) * rho;
+}
+
+struct Nb {
+    double u[5];
+    double rho, sq;
+};
+
+__device__ __forceinline__ Nb load_nb(const double *su, const double2 *sa, int uidx, int aidx) {
+    Nb n;
+#pragma unroll
+    for (int m = 0; m < 5; ++m) n.u[m] = su[m * UPM + uidx];
+    const double2 a = sa[aidx];
+    n.rho = a.x;
+    n.sq = a.y;
+    return n;
+}
+
+__device__ __forceinline__ void load5(double (&a)[5], const double *su, int uidx) {
+#pragma unroll
+    for (int m = 0; m < 5; ++m) a[m] = su[m * UPM + uidx];
+}
+
+// Flux differences along one axis (App. A steps 2 / 4 / 6).  MOM = index of
+// the momentum component along the axis (1 = xi, 2 = eta, 3 = zeta).
+template <int MOM>
+__device__ __forceinline__ void flux_dir(double (&acc)[5], const double (&cu)[5],
+                                         const double (&vc)[3], double qsc, double pc,
+                                         const Nb &p, const Nb &q, const Coef &C, int ax) {
+    double vp[3], vq[3];
+#pragma unroll
+    for (int n = 0; n < 3; ++n) {
+        vp[n] = p.u[n + 1] * p.rho;
+        vq[n] = q.u[n + 1] * q.rho;
+    }
+    const double wp = vp[MOM - 1], wq = vq[MOM - 1], wc = vc[MOM - 1];
+    const double t2 = C.t2[ax];
+
+    acc[0] = acc[0] + C.d1[ax][0] * d2(p.u[0], cu[0], q.u[0]);
+    acc[0] = acc[0] - t2 * (p.u[MOM] - q.u[MOM]);
+#pragma unroll
+    for (int m = 1; m <= 3; ++m) {
+        acc[m] = acc[m] + C.d1[ax][m] * d2(p.u[m], cu[m], q.u[m]);
+        if (m == MOM) {
+            acc[m] = acc[m] + C.con2x43[ax] * d2(wp, wc, wq);
+            acc[m] = acc[m] - t2 * ((p.u[m] * wp - q.u[m] * wq) +
+                                    (((p.u[4] - p.sq) - q.u[4]) + q.sq) * C.c2);
+        } else {
+            acc[m] = acc[m] + C.con2[ax] * d2(vp[m - 1], vc[m - 1], vq[m - 1]);
+            acc[m] = acc[m] - t2 * (p.u[m] * wp - q.u[m] * wq);
+        }
+    }
+    acc[4] = acc[4] + C.d1[ax][4] * d2(p.u[4], cu[4], q.u[4]);
+    acc[4] = acc[4] + C.con3[ax] * d2(p.sq * p.rho, qsc, q.sq * q.rho);
+    acc[4] = acc[4] + C.con4[ax] * d2(wp * wp, wc * wc, wq * wq);
+    acc[4] = acc[4] + C.con5[ax] * d2(p.u[4] * p.rho, pc, q.u[4] * q.rho);
+    acc[4] = acc[4] - t2 * ((C.c1 * p.u[4] - C.c2 * p.sq) * wp -
+                            (C.c1 * q.u[4] - C.c2 * q.sq) * wq);
+}
+
+// Fourth-order dissipation along one axis (App. A steps 3 / 5 / 7).  The
+// GENERIC form covers all five NAS cases by zero-selecting the absent
+// neighbours (exact: 0 - 4a = -4a, x + 0 = x) and choosing 5.0 or 6.0 for
+// the centre; the non-generic form is the interior case only.
+struct Cases {
+    bool hm2, hm1, hp1, hp2, five;
+};
+
+__device__ __forceinline__ Cases cases_of(int x, int n) {
+    Cases c;
+    c.hm2 = x >= 3;
+    c.hm1 = x >= 2;
+    c.hp1 = x <= n - 3;
+    c.hp2 = x <= n - 4;
+    c.five = (x == 1) || (x == n - 2);
+    return c;
+}
+
+__device__ __forceinline__ bool is_mid(int x, int n) { return x >= 3 && x <= n - 4; }
+
+template <bool GENERIC>
+__device__ __forceinline__ void diss_dir(double (&acc)[5], const double (&am2)[5],
+                                         const double (&am1)[5], const double (&a0)[5],
+                                         const double (&six)[5], const double (&ap1)[5],
+                                         const double (&ap2)[5], double dssp, Cases cs) {
+#pragma unroll
+    for (int m = 0; m < 5; ++m) {
+        double t;
+        if (!GENERIC) {
+            t = __fma_rn(-4.0, am1[m], am2[m]);
+            t = t + six[m];
+            t = __fma_rn(-4.0, ap1[m], t);
+            t = t + ap2[m];
+        } else {
+            const double x2 = cs.hm2 ? am2[m] : 0.0;
+            const double x1 = cs.hm1 ? am1[m] : 0.0;
+            const double y1 = cs.hp1 ? ap1[m] : 0.0;
+            const double y2 = cs.hp2 ? ap2[m] : 0.0;
+            const double cc = cs.five ? 5.0 * a0[m] : six[m];
+            t = __fma_rn(-4.0, x1, x2);
+            t = t + cc;
+            t = __fma_rn(-4.0, y1, t);
+            t = t + y2;
+        }
+        acc[m] = acc[m] - dssp * t;
+    }
+}
+
+// Copy forcing -> rhs on this launch's boundary-face points (rhs = forcing,
+// unscaled; App. A step 1, reading c3), spread over all CTAs.
+__device__ __forceinline__ void copy_faces(const Params &P) {
+    const int nx = P.nx, ny = P.ny;
+    const int per = 2 * nx + 2 * (ny - 2);
+    const int nloc = P.fk_hi - P.fk_lo;
+    if (nloc <= 0) return;
+    const long long nper = (long long)per * nloc;
+    // full planes: global k == 0 or nz-1 inside [fk_lo, fk_hi)
+    const int kl0 = 0 - P.k0, kl1 = (P.nz - 1) - P.k0;
+    const bool has0 = kl0 >= P.fk_lo && kl0 < P.fk_hi;
+    const bool has1 = kl1 >= P.fk_lo && kl1 < P.fk_hi;
+    const int nfull = (int)has0 + (int)has1;
+    const int full0 = has0 ? kl0 : kl1;  // first full plane; the second is always kl1
+    const long long inner = (long long)(nx - 2) * (ny - 2);
+    const long long total = nper + inner * nfull;
+    const long long stride = (long long)gridDim.x * blockDim.x;
+    for (long long t = (long long)blockIdx.x * blockDim.x + threadIdx.x; t < total; t += stride) {
+        int i, j, kl;
+        if (t < nper) {
+            kl = P.fk_lo + (int)(t / per);
+            int e = (int)(t % per);
+            if (e < nx) {
+                i = e; j = 0;
+            } else if (e < 2 * nx) {
+                i = e - nx; j = ny - 1;
+            } else {
+                e -= 2 * nx;
+                if (e < ny - 2) { i = 0; j = 1 + e; }
+                else { i = nx - 1; j = 1 + e - (ny - 2); }
+            }
+        } else {
+            const long long e = t - nper;
+            kl = (e < inner) ? full0 : kl1;
+            const int r = (int)(e % inner);
+            i = 1 + r % (nx - 2);
+            j = 1 + r / (nx - 2);
+        }
+        const int o = i + P.sy * j + P.sk * kl;
+#pragma unroll
+        for (int m = 0; m < 5; ++m) __stcs(P.r + o + P.sm * m, __ldcs(P.f + o + P.sm * m));
+    }
+}
+
+__device__ __forceinline__ void issue_plane(const CUtensorMap *tmap, const Params &P,
+                                            double *su, uint64_t *mbar, int i0, int j0, int k,
+                                            uint32_t seq) {
+    const int slot = (int)(seq % STAGES);
+    const int kb = k - P.k0 + P.ukoff;
+    const int jc = j0 - 2;
+    const int c1 = P.pos_j == 1 ? jc : (P.pos_m == 1 ? 0 : kb);
+    const int c2 = P.pos_j == 2 ? jc : (P.pos_m == 2 ? 0 : kb);
+    const int c3 = P.pos_j == 3 ? jc : (P.pos_m == 3 ? 0 : kb);
+    mbar_expect_tx(&mbar[slot], TMA_BYTES);
+    tma_load_4d(su + (size_t)slot * U_PLANE, tmap, &mbar[slot], i0 - 2, c1, c2, c3);
+}
+
+__device__ __forceinline__ void wait_plane(uint64_t *mbar, uint32_t seq) {
+    mbar_wait(&mbar[seq % STAGES], (seq / STAGES) & 1u);
+}
+
+// One CTA processes the column-plane units [blockIdx*units/ncta, ...).
+__device__ __forceinline__ void rhs_body(const CUtensorMap *tmap, const Params &P) {
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    double *su = reinterpret_cast<double *>(smem_raw);
+    double2 *sa = reinterpret_cast<double2 *>(su + (size_t)STAGES * U_PLANE);
+    uint64_t *mbar = reinterpret_cast<uint64_t *>(sa + (size_t)AUX_SLOTS * A_PLANE);
+
+    const int tid = threadIdx.x;
+    const int tx = tid % TX, ty = tid / TX;
+    const Coef &C = P.c;
+
+    if (tid == 0) {
+        prefetch_tmap(tmap);
+        for (int s = 0; s < STAGES; ++s) mbar_init(&mbar[s], 1);
+        fence_mbar_init();
+    }
+    __syncthreads();
+
+    copy_faces(P);
+
+    long long ub = (long long)blockIdx.x * P.units / P.ncta;
+    const long long ue = (long long)(blockIdx.x + 1) * P.units / P.ncta;
+    uint32_t seq0 = 0;
+
+    while (ub < ue) {
+        // ---- segment: one column tile, a contiguous run of planes ----
+        const int col = (int)(ub / P.nplanes);
+        const int pidx = (int)(ub % P.nplanes);
+        int ka, kb;
+        {
+            const long long left = ue - ub;
+            if (pidx < P.n0) {
+                ka = P.ka0 + pidx;
+                kb = (int)min((long long)P.kb0, ka + left);
+            } else {
+                ka = P.ka1 + (pidx - P.n0);
+                kb = (int)min((long long)P.kb1, ka + left);
+            }
+        }
+        ub += kb - ka;
+
+        const int i0 = 1 + (col % P.ntx) * TX;
+        const int j0 = 1 + (col / P.ntx) * TY;
+        const int i = i0 + tx, j = j0 + ty;
+        const bool in_grid = (i < P.nx) && (j < P.ny);
+        const bool active = (i <= P.nx - 2) && (j <= P.ny - 2);
+        const int nload = kb - ka + 2;  // planes ka .. kb+1
+
+        if (tid == 0) {
+            const int npre = nload < STAGES ? nload : STAGES;
+            for (int s = 0; s < npre; ++s) issue_plane(tmap, P, su, mbar, i0, j0, ka + s, seq0 + s);
+        }
+
+        // Case flags (global indices, reading c12).
+        const bool mid_x = is_mid(i0, P.nx) && is_mid(i0 + TX - 1, P.nx);
+        const bool mid_y = is_mid(j, P.ny);
+        const Cases cx = cases_of(i, P.nx), cy = cases_of(j, P.ny);
+
+        const int uc = (ty + 2) * UX + (tx + 2);   // centre in the u tile
+        const int ac = (ty + 1) * AX + (tx + 1);   // centre in the aux tile
+        const int ocol = i + P.sy * j;             // own column offset (dim)
+
+        // Register window u(:, k-2..k+2) and own rho_i/square at k-1..k+1.
+        double w0[5], w1[5], w2[5], w3[5], w4[5];
+        double rm1, sm1, r0, s0, rp1, sp1;
+        {
+            const int kbm2 = ka - 2 - P.k0 + P.ukoff, kbm1 = ka - 1 - P.k0 + P.ukoff;
+#pragma unroll
+            for (int m = 0; m < 5; ++m) {
+                w0[m] = (in_grid && kbm2 >= 0) ? __ldg(P.u + ocol + P.sm * m + P.sk * kbm2) : 0.0;
+                w1[m] = (in_grid && kbm1 >= 0) ? __ldg(P.u + ocol + P.sm * m + P.sk * kbm1) : 0.0;
+            }
+            if (in_grid && kbm1 >= 0) aux_of(w1[0], w1[1], w1[2], w1[3], rm1, sm1);
+            else { rm1 = 0.0; sm1 = 0.0; }
+        }
+        // plane ka: own column, own aux, ring aux
+        wait_plane(mbar, seq0);
+        {
+            const double *s = su + (size_t)((seq0) % STAGES) * U_PLANE;
+            double2 *a = sa + (size_t)(ka % AUX_SLOTS) * A_PLANE;
+            load5(w2, s, uc);
+            if (in_grid) aux_of(w2[0], w2[1], w2[2], w2[3], r0, s0);
+            else { r0 = 0.0; s0 = 0.0; }
+            a[ac] = make_double2(r0, s0);
+            if (tid < NRING) {
+                int ii, jj;
+                if (tid < AX) { ii = tid; jj = 0; }
+                else if (tid < 2 * AX) { ii = tid - AX; jj = AY - 1; }
+                else if (tid < 2 * AX + TY) { ii = 0; jj = 1 + tid - 2 * AX; }
+                else { ii = AX - 1; jj = 1 + tid - 2 * AX - TY; }
+                const int gi = i0 - 1 + ii, gj = j0 - 1 + jj;
+                double rr = 0.0, ss = 0.0;
+                if (gi >= 0 && gi < P.nx && gj >= 0 && gj < P.ny) {
+                    const int ui = (jj + 1) * UX + (ii + 1);
+                    aux_of(s[ui], s[UPM + ui], s[2 * UPM + ui], s[3 * UPM + ui], rr, ss);
+                }
+                a[jj * AX + ii] = make_double2(rr, ss);
+            }
+        }
+        wait_plane(mbar, seq0 + 1);
+        load5(w3, su + (size_t)((seq0 + 1) % STAGES) * U_PLANE, uc);
+
+        for (int k = ka; k < kb; ++k) {
+            const uint32_t sq_k = seq0 + (uint32_t)(k - ka);
+            // (0) stream forcing(k): used once, never staged (reuse count 1)
+            double fr[5];
+            {
+                const int kl = k - P.k0;
+#pragma unroll
+                for (int m = 0; m < 5; ++m)
+                    fr[m] = active ? __ldcs(P.f + ocol + P.sm * m + P.sk * kl) : 0.0;
+            }
+            // (1) own column u(k+2) into the window
+            wait_plane(mbar, sq_k + 2);
+            load5(w4, su + (size_t)((sq_k + 2) % STAGES) * U_PLANE, uc);
+            // (2) rho_i / square of plane k+1: own point (registers + smem) and halo ring
+            {
+                if (in_grid) aux_of(w3[0], w3[1], w3[2], w3[3], rp1, sp1);
+                else { rp1 = 0.0; sp1 = 0.0; }
+                double2 *a = sa + (size_t)((k + 1) % AUX_SLOTS) * A_PLANE;
+                a[ac] = make_double2(rp1, sp1);
+                if (k + 1 < kb && tid < NRING) {
+                    const double *s = su + (size_t)((sq_k + 1) % STAGES) * U_PLANE;
+                    int ii, jj;
+                    if (tid < AX) { ii = tid; jj = 0; }
+                    else if (tid < 2 * AX) { ii = tid - AX; jj = AY - 1; }
+                    else if (tid < 2 * AX + TY) { ii = 0; jj = 1 + tid - 2 * AX; }
+                    else { ii = AX - 1; jj = 1 + tid - 2 * AX - TY; }
+                    const int gi = i0 - 1 + ii, gj = j0 - 1 + jj;
+                    double rr = 0.0, ss = 0.0;
+                    if (gi >= 0 && gi < P.nx && gj >= 0 && gj < P.ny) {
+                        const int ui = (jj + 1) * UX + (ii + 1);
+                        aux_of(s[ui], s[UPM + ui], s[2 * UPM + ui], s[3 * UPM + ui], rr, ss);
+                    }
+                    a[jj * AX + ii] = make_double2(rr, ss);
+                }
+            }
+            __syncthreads();
+            // (3) refill the slot plane k-1 used (every thread is past step k-1)
+            if (tid == 0 && k > ka) {
+                const int kn = k - 1 + STAGES;
+                if (kn <= kb + 1) issue_plane(tmap, P, su, mbar, i0, j0, kn, sq_k - 1 + STAGES);
+            }
+            // (5) the point (i, j, k)
+            if (active) {
+                const double *s = su + (size_t)(sq_k % STAGES) * U_PLANE;
+                const double2 *a = sa + (size_t)(k % AUX_SLOTS) * A_PLANE;
+
+                double acc[5];
+#pragma unroll
+                for (int m = 0; m < 5; ++m) acc[m] = fr[m];
+
+                double vc[3];
+                vc[0] = w2[1] * r0;
+                vc[1] = w2[2] * r0;
+                vc[2] = w2[3] * r0;
+                const double qsc = s0 * r0;
+                const double pc = w2[4] * r0;
+                double six[5];
+#pragma unroll
+                for (int m = 0; m < 5; ++m) six[m] = 6.0 * w2[m];
+
+                // xi
+                {
+                    const Nb p = load_nb(s, a, uc + 1, ac + 1);
+                    const Nb q = load_nb(s, a, uc - 1, ac - 1);
+                    flux_dir<1>(acc, w2, vc, qsc, pc, p, q, C, 0);
+                    double pp[5], qq[5];
+                    load5(pp, s, uc + 2);
+                    load5(qq, s, uc - 2);
+                    if (mid_x) diss_dir<false>(acc, qq, q.u, w2, six, p.u, pp, C.dssp, cx);
+                    else diss_dir<true>(acc, qq, q.u, w2, six, p.u, pp, C.dssp, cx);
+                }
+                // eta
+                {
+                    const Nb p = load_nb(s, a, uc + UX, ac + AX);
+                    const Nb q = load_nb(s, a, uc - UX, ac - AX);
+                    flux_dir<2>(acc, w2, vc, qsc, pc, p, q, C, 1);
+                    double pp[5], qq[5];
+                    load5(pp, s, uc + 2 * UX);
+                    load5(qq, s, uc - 2 * UX);
+                    if (mid_y) diss_dir<false>(acc, qq, q.u, w2, six, p.u, pp, C.dssp, cy);
+                    else diss_dir<true>(acc, qq, q.u, w2, six, p.u, pp, C.dssp, cy);
+                }
+                // zeta: everything from the register window
+                {
+                    Nb p, q;
+#pragma unroll
+                    for (int m = 0; m < 5; ++m) {
+                        p.u[m] = w3[m];
+                        q.u[m] = w1[m];
+                    }
+                    p.rho = rp1; p.sq = sp1;
+                    q.rho = rm1; q.sq = sm1;
+                    flux_dir<3>(acc, w2, vc, qsc, pc, p, q, C, 2);
+                    if (is_mid(k, P.nz)) diss_dir<false>(acc, w0, w1, w2, six, w3, w4, C.dssp, Cases{});
+                    else diss_dir<true>(acc, w0, w1, w2, six, w3, w4, C.dssp, cases_of(k, P.nz));
+                }
+                const int o = ocol + P.sk * (k - P.k0);
+#pragma unroll
+                for (int m = 0; m < 5; ++m) __stcs(P.r + o + P.sm * m, acc[m] * C.dt);
+            }
+            // (6) rotate the windows
+#pragma unroll
+            for (int m = 0; m < 5; ++m) {
+                w0[m] = w1[m];
+                w1[m] = w2[m];
+                w2[m] = w3[m];
+                w3[m] = w4[m];
+            }
+            rm1 = r0; sm1 = s0;
+            r0 = rp1; s0 = sp1;
+        }
+        seq0 += (uint32_t)nload;
+        __syncthreads();  // every slot / aux plane of this segment is consumed
+    }
+}
+
+}  // namespace dev
+}  // namespace safara

@@ -1,0 +1,67 @@
+// safara_internal.h -- types shared by the host ABI (api.cu) and the kernel
+// translation units (rhs_fast.cu / rhs_strict.cu).  Not part of the C ABI.
+#pragma once
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "safara.h"
+
+namespace safara {
+
+// CTA tile: TX x TY (i, j) columns, one thread per column marching along k.
+constexpr int TX = 32;
+#ifndef SAFARA_TY
+#define SAFARA_TY 10
+#endif
+constexpr int TY = SAFARA_TY;
+constexpr int NTHREADS = TX * TY;
+constexpr int STAGES = 5;            // u planes in the TMA ring
+constexpr int UX = TX + 4;           // u tile incl. i halo of 2
+constexpr int UY = TY + 4;           // u tile incl. j halo of 2
+constexpr int AX = TX + 2;           // aux (rho_i, square) tile incl. halo of 1
+constexpr int AY = TY + 2;
+constexpr int AUX_SLOTS = 3;         // aux planes k, k+1 (being written), k+2
+constexpr int U_PLANE = UX * UY * 5; // doubles per ring slot (one TMA box)
+constexpr int A_PLANE = AX * AY;     // double2 {rho_i, square} per aux slot
+constexpr int NRING = 2 * AX + 2 * TY;  // aux halo points recomputed per plane
+constexpr uint32_t TMA_BYTES = U_PLANE * 8u;
+constexpr size_t SMEM_BYTES =
+    (size_t)STAGES * U_PLANE * 8 + (size_t)AUX_SLOTS * A_PLANE * 16 + STAGES * 8;
+constexpr int MIN_PLANES_PER_CTA = 4;
+
+// Device-side coefficients: safara_coeffs_t plus the constant products that
+// the NAS text evaluates left to right (xxcon2*con43 -> one double).
+struct Coef {
+    double dt, dssp, c1, c2;
+    double t2[3];          // tx2, ty2, tz2
+    double d1[3][5];       // dx{m}tx1, dy{m}ty1, dz{m}tz1
+    double con2[3], con2x43[3], con3[3], con4[3], con5[3];
+};
+
+struct Params {
+    int nx, ny, nz;        // global extents
+    int sy, sm, sk;        // shared element strides (dim clause), int32 (small)
+    int k0;                // global k of forcing/rhs local plane 0
+    int ukoff;             // u local plane = k - k0 + ukoff
+    int nzu;               // planes in the u buffer
+    int ka0, kb0, ka1, kb1;// global planes to compute: [ka0,kb0) U [ka1,kb1)
+    int n0, nplanes;       // n0 = kb0-ka0, nplanes = n0 + (kb1-ka1)
+    int ntx, nty;          // column tiles
+    int ncta;              // CTAs in the grid
+    long long units;       // ntx*nty*nplanes (column-plane work items)
+    int fk_lo, fk_hi;      // local planes whose boundary faces this launch copies
+    int pos_j, pos_m, pos_k;  // tensor-map dimension holding j, m, k
+    const double *u;       // u buffer base (local plane 0)
+    const double *f;       // forcing base (local plane 0)
+    double *r;             // rhs base (local plane 0)
+    Coef c;
+};
+
+// Launchers implemented in rhs_fast.cu / rhs_strict.cu.
+cudaError_t launch_rhs_fast(const CUtensorMap &tmap, const Params &p, cudaStream_t s);
+cudaError_t launch_rhs_strict(const CUtensorMap &tmap, const Params &p, cudaStream_t s);
+cudaError_t setup_rhs_fast(int *ctas_per_sm, cudaFuncAttributes *attr);
+cudaError_t setup_rhs_strict(int *ctas_per_sm, cudaFuncAttributes *attr);
+
+}  // namespace safara

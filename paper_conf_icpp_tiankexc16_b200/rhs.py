@@ -1,0 +1,142 @@
+"""Torch-facing wrappers of the C ABI (argument marshalling only).
+
+Canonical layout (include/safara.h): a field is a float64
+tensor of shape ``(nz, 5, ny, sy)`` with ``sy = pitch(nx)``; element
+(i, j, m, k) sits at offset ``i + sy*j + sm*m + sk*k``.  ``pack``/``unpack``
+convert from/to the logical ``(nz, ny, nx, 5)`` layout used by ``nasgen`` and
+the oracle; they are input/output marshalling, not part of the pass.
+"""
+from __future__ import annotations
+
+import ctypes
+
+import numpy as np
+import torch
+
+from ._abi import (SAFARA_FLAG_STRICT, SAFARA_PART_ALL, Coeffs, Dims, KernelInfo,
+                   check, lib)
+
+_initialised: set[int] = set()
+
+
+def init(device: int | None = None) -> int:
+    """safara_rhs_init for ``device`` (default: current CUDA device)."""
+    if device is None:
+        device = torch.cuda.current_device()
+    if device not in _initialised:
+        check(lib().safara_rhs_init(int(device)), "safara_rhs_init")
+        _initialised.add(device)
+    return device
+
+
+def pitch(nx: int) -> int:
+    return lib().safara_pitch(int(nx))
+
+
+def canonical_dims(nx: int, ny: int, nz: int) -> Dims:
+    d = Dims()
+    check(lib().safara_dims_canonical(nx, ny, nz, ctypes.byref(d)), "safara_dims_canonical")
+    return d
+
+
+def validate_dims(d: Dims, nz_buf: int) -> int:
+    return lib().safara_validate_dims(ctypes.byref(d), int(nz_buf))
+
+
+def coeffs_nas(nx: int, ny: int, nz: int, dt: float) -> Coeffs:
+    c = Coeffs()
+    check(lib().safara_coeffs_nas(nx, ny, nz, float(dt), ctypes.byref(c)), "safara_coeffs_nas")
+    return c
+
+
+def empty_field(nx: int, ny: int, nplanes: int, device="cuda", pin: bool = False) -> torch.Tensor:
+    """Uninitialised canonical field of ``nplanes`` k-planes."""
+    t = torch.empty((nplanes, 5, ny, pitch(nx)), dtype=torch.float64,
+                    device="cpu" if pin else device, pin_memory=pin)
+    return t
+
+
+def pack(a, device="cuda", pin: bool = False) -> torch.Tensor:
+    """Logical (nz, ny, nx, 5) array -> canonical (nz, 5, ny, sy) tensor
+    (pitch padding zero-filled)."""
+    t = torch.as_tensor(np.ascontiguousarray(a) if isinstance(a, np.ndarray) else a,
+                        dtype=torch.float64)
+    nz, ny, nx, five = t.shape
+    assert five == 5
+    out = torch.zeros((nz, 5, ny, pitch(nx)), dtype=torch.float64,
+                      device="cpu" if pin else device, pin_memory=pin)
+    out[..., :nx] = t.permute(0, 3, 1, 2).to(out.device)
+    return out
+
+
+def unpack(t: torch.Tensor, nx: int) -> np.ndarray:
+    """Canonical (nz, 5, ny, sy) tensor -> logical (nz, ny, nx, 5) numpy array."""
+    return np.ascontiguousarray(t[..., :nx].permute(0, 2, 3, 1).cpu().numpy())
+
+
+def _stream_ptr(stream) -> int | None:
+    if stream is None:
+        stream = torch.cuda.current_stream()
+    return stream.cuda_stream if hasattr(stream, "cuda_stream") else int(stream)
+
+
+def _check_field(t: torch.Tensor, name: str):
+    if t.dtype != torch.float64 or not t.is_cuda or not t.is_contiguous():
+        raise ValueError(f"{name} must be a contiguous float64 CUDA tensor")
+
+
+def rhs(u: torch.Tensor, forcing: torch.Tensor, out: torch.Tensor, nx: int, coeffs: Coeffs,
+        strict: bool = False, stream=None, dims: Dims | None = None) -> torch.Tensor:
+    """One compute_rhs pass: ``out <- F(u, forcing)`` on the GPU (async).
+
+    Tensors are canonical ``(nz, 5, ny, sy)`` unless ``dims`` describes
+    another stride order (then they are flat buffers of that layout)."""
+    for t, n in ((u, "u"), (forcing, "forcing"), (out, "out")):
+        _check_field(t, n)
+    if dims is None:
+        nz, _, ny, _ = u.shape
+        dims = canonical_dims(nx, ny, nz)
+    flags = SAFARA_FLAG_STRICT if strict else 0
+    check(lib().safara_rhs_ex(u.data_ptr(), forcing.data_ptr(), out.data_ptr(),
+                              ctypes.byref(dims), ctypes.byref(coeffs), flags,
+                              _stream_ptr(stream)), "safara_rhs_ex")
+    return out
+
+
+def rhs_slab(u_slab: torch.Tensor, forcing_slab: torch.Tensor, out_slab: torch.Tensor,
+             nx: int, nz: int, k0: int, coeffs: Coeffs, part: int = SAFARA_PART_ALL,
+             strict: bool = False, stream=None) -> torch.Tensor:
+    """z-slab pass: u_slab has nzl+4 planes (2 ghosts each side), forcing /
+    out have nzl planes; this slab owns global planes [k0, k0+nzl)."""
+    for t, n in ((u_slab, "u_slab"), (forcing_slab, "forcing_slab"), (out_slab, "out_slab")):
+        _check_field(t, n)
+    nzl, _, ny, _ = forcing_slab.shape
+    dims = canonical_dims(nx, ny, nz)
+    flags = SAFARA_FLAG_STRICT if strict else 0
+    check(lib().safara_rhs_slab(u_slab.data_ptr(), forcing_slab.data_ptr(), out_slab.data_ptr(),
+                                ctypes.byref(dims), int(k0), int(nzl), ctypes.byref(coeffs),
+                                flags, int(part), _stream_ptr(stream)), "safara_rhs_slab")
+    return out_slab
+
+
+def rhs_host(u_host: torch.Tensor, f_host: torch.Tensor, r_host: torch.Tensor,
+             u_dev: torch.Tensor, f_dev: torch.Tensor, r_dev: torch.Tensor, nx: int,
+             coeffs: Coeffs, strict: bool = False, nchunks: int = 1, stream=None):
+    """End-to-end pass on host (pinned) canonical tensors through device buffers."""
+    nz, _, ny, _ = u_host.shape
+    flags = SAFARA_FLAG_STRICT if strict else 0
+    check(lib().safara_rhs_host(u_host.data_ptr(), f_host.data_ptr(), r_host.data_ptr(),
+                                u_dev.data_ptr(), f_dev.data_ptr(), r_dev.data_ptr(),
+                                nx, ny, nz, ctypes.byref(coeffs), flags, int(nchunks),
+                                _stream_ptr(stream)), "safara_rhs_host")
+    return r_host
+
+
+def launch_count() -> int:
+    return int(lib().safara_launch_count())
+
+
+def kernel_info(strict: bool = False) -> dict:
+    k = KernelInfo()
+    check(lib().safara_kernel_info(1 if strict else 0, ctypes.byref(k)), "safara_kernel_info")
+    return {f: getattr(k, f) for f, _ in KernelInfo._fields_}

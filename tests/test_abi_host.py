@@ -1,0 +1,108 @@
+"""Host-side checks of the C ABI that need no GPU: the library builds for
+sm_100a, loads, exports every symbol include/safara.h declares, and its host
+logic (descriptor validation = the dim/small clause check, PAPER.md
+L1275-1291; NPB coefficients; canonical pitch) behaves as documented."""
+import ctypes
+import subprocess
+
+import pytest
+
+import paper_conf_icpp_tiankexc16_b200 as sr
+from paper_conf_icpp_tiankexc16_b200 import _abi, build
+
+
+@pytest.fixture(scope="module")
+def L():
+    build.build()
+    return _abi.lib()
+
+
+def test_exports_every_header_symbol(L):
+    syms = _abi.header_symbols()
+    assert len(syms) >= 12
+    for s in syms:
+        assert hasattr(L, s), s
+    out = subprocess.run(["nm", "-D", "--defined-only", _abi.LIB_PATH], capture_output=True,
+                         text=True).stdout
+    for s in syms:
+        assert f" T {s}" in out, s
+
+
+def test_sass_is_sm100a_with_tma():
+    build.build()
+    sass = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "-sass", _abi.LIB_PATH],
+                          capture_output=True, text=True).stdout
+    assert "sm_100a" in sass
+    assert "UTMALDG" in sass          # cp.async.bulk.tensor (TMA) loads
+    assert "DFMA" in sass and "DMUL" in sass
+    assert "HMMA" not in sass         # no legacy tensor-core path
+
+
+def test_ptxas_zero_spills():
+    build.build(force=True)
+    log = open(build.os.path.join(build.BUILD, "ptxas.txt")).read()
+    assert log.count("0 bytes spill stores, 0 bytes spill loads") >= 2, log
+    assert "0 bytes stack frame" in log
+
+
+def test_pitch_and_canonical_dims(L):
+    for nx, p in ((12, 16), (36, 40), (64, 64), (102, 104), (162, 168)):
+        assert sr.pitch(nx) == p
+        d = sr.canonical_dims(nx, nx, nx)
+        assert (d.sy, d.sm, d.sk) == (p, nx * p, 5 * nx * p)
+        assert sr.validate_dims(d, nx) == 0
+
+
+def test_validation_errors(L):
+    d = sr.canonical_dims(12, 12, 12)
+    assert sr.validate_dims(d, 12) == 0
+    bad = _abi.Dims(5, 12, 12, d.sy, d.sm, d.sk)
+    assert sr.validate_dims(bad, 12) == -2                     # SHAPE: n < 6
+    bad = _abi.Dims(12, 12, 12, 10, d.sm, d.sk)
+    assert sr.validate_dims(bad, 12) == -3                     # LAYOUT: sy < nx
+    bad = _abi.Dims(12, 12, 12, 16, 100, d.sk)
+    assert sr.validate_dims(bad, 12) == -3                     # LAYOUT: m overlaps j
+    bad = _abi.Dims(12, 12, 12, 13, 13 * 12, 13 * 60)
+    assert sr.validate_dims(bad, 12) == -4                     # ALIGN: odd stride
+    big = sr.canonical_dims(1000, 1000, 20)
+    assert sr.validate_dims(big, 20) == 0
+    assert sr.validate_dims(big, 500) == -5                    # TOO_LARGE: small is false
+    # SP-native [m][k][j][i]: k stride below m stride is a valid descriptor.
+    nx = ny = nz = 12
+    sp = _abi.Dims(nx, ny, nz, 16, 16 * ny * nz, 16 * ny)
+    assert sr.validate_dims(sp, nz) == 0
+
+
+def test_canonical_too_large(L):
+    d = _abi.Dims()
+    assert L.safara_dims_canonical(2000, 2000, 200, ctypes.byref(d)) == -5
+
+
+def test_strerror(L):
+    for code in range(0, -9, -1):
+        assert len(_abi.strerror(code)) > 5
+    assert "unknown" in _abi.strerror(-99)
+
+
+def test_coeffs_match_nas_constants(L):
+    """The library's own set_constants equals the oracle's, value for value
+    (both follow SURVEY App. B; they share no code)."""
+    import oracle
+    for n, dt in ((12, 0.01), (36, 0.0015), (162, 0.0001)):
+        c = sr.coeffs_nas(n, n + 2, n + 4, dt)
+        o = oracle.set_constants(n, n + 2, n + 4, dt)
+        assert c.dt == o.dt and c.dssp == o.dssp and c.c1 == o.c1 and c.c2 == o.c2
+        assert c.con43 == o.con43
+        assert (c.tx2, c.ty2, c.tz2) == (o.tx2, o.ty2, o.tz2)
+        for m in range(5):
+            assert c.dxt[m] == getattr(o, f"dx{m + 1}tx1")
+            assert c.dyt[m] == getattr(o, f"dy{m + 1}ty1")
+            assert c.dzt[m] == getattr(o, f"dz{m + 1}tz1")
+            for ax in ("xx", "yy", "zz"):
+                assert getattr(c, ax + "con")[m] == getattr(o, f"{ax}con{m + 1}")
+
+
+def test_compute_without_init_fails_loudly(L):
+    # No GPU here: the compute entry must return an error, never run on the CPU.
+    rc = L.safara_rhs(1 << 20, 2 << 20, 3 << 20, 12, 12, 12, ctypes.byref(_abi.Coeffs()), None)
+    assert rc < 0

@@ -1,0 +1,196 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle.
+
+Bar: STRICT variant bit-identical to the oracle; production
+variant within |g - o| <= 1e-12 |o| + 1e-14 elementwise (BASELINE.json
+north_star, reading c5).  Inputs: nasgen (exact solution x (1 + 1e-3 noise),
+forcing = exact_rhs [+ noise]), identical on both sides.
+"""
+import numpy as np
+import pytest
+import torch
+
+import nasgen
+import oracle
+import paper_conf_icpp_tiankexc16_b200 as sr
+
+pytestmark = pytest.mark.gpu
+
+RTOL, ATOL = 1e-12, 1e-14
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _init():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    sr.init(0)
+
+
+def gpu_rhs(u, f, dt, strict, nx=None):
+    nz, ny, nx_, _ = u.shape
+    nx = nx_ if nx is None else nx
+    du, df = sr.pack(u), sr.pack(f)
+    dr = torch.full_like(du, float("nan"))
+    c = sr.coeffs_nas(nx, ny, nz, dt)
+    n0 = sr.launch_count()
+    sr.rhs(du, df, dr, nx, c, strict=strict)
+    torch.cuda.synchronize()
+    assert sr.launch_count() == n0 + 1
+    return sr.unpack(dr, nx)
+
+
+def assert_tol(g, o):
+    err = np.abs(g - o)
+    bound = RTOL * np.abs(o) + ATOL
+    bad = err > bound
+    assert not bad.any(), (f"{bad.sum()} elements out of tolerance; worst ratio "
+                           f"{(err / bound).max():.3g}")
+
+
+def oracle_rhs(inp):
+    return oracle.compute_rhs(inp.u, inp.forcing, dt=inp.dt, threads=8)
+
+
+SMALL = [("BT", "S"), ("SP", "W"), ("BT", "W"), ("BT", "A")]
+
+
+@pytest.mark.parametrize("bench,cls", SMALL)
+def test_strict_bitwise_classes(bench, cls):
+    inp = nasgen.make_class(bench, cls, seed=1, B=1e-2)
+    o = oracle_rhs(inp)
+    g = gpu_rhs(inp.u, inp.forcing, inp.dt, strict=True)
+    assert np.array_equal(g, o), f"max |g-o| = {np.abs(g - o).max():.3g}"
+
+
+@pytest.mark.parametrize("shape", [(6, 6, 6), (7, 7, 7), (9, 13, 37), (17, 29, 37),
+                                   (11, 70, 41), (8, 12, 66), (23, 15, 100)])
+def test_strict_bitwise_ragged(shape):
+    nz, ny, nx = shape
+    inp = nasgen.make_inputs(nx, ny, nz, seed=2, B=1e-2, dt=0.003)
+    o = oracle_rhs(inp)
+    g = gpu_rhs(inp.u, inp.forcing, inp.dt, strict=True)
+    assert np.array_equal(g, o), f"max |g-o| = {np.abs(g - o).max():.3g}"
+
+
+@pytest.mark.parametrize("bench,cls", SMALL + [("SP", "B"), ("BT", "C")])
+def test_fast_within_tolerance(bench, cls):
+    inp = nasgen.make_class(bench, cls, seed=3)
+    o = oracle_rhs(inp)
+    g = gpu_rhs(inp.u, inp.forcing, inp.dt, strict=False)
+    assert_tol(g, o)
+    faces = np.ones(o.shape[:3], dtype=bool)
+    faces[1:-1, 1:-1, 1:-1] = False
+    assert np.array_equal(g[faces], inp.forcing[faces])
+
+
+@pytest.mark.parametrize("bench,cls", [("SP", "B"), ("BT", "C")])
+def test_strict_bitwise_large(bench, cls):
+    inp = nasgen.make_class(bench, cls, seed=1)
+    o = oracle_rhs(inp)
+    g = gpu_rhs(inp.u, inp.forcing, inp.dt, strict=True)
+    assert np.array_equal(g, o)
+
+
+def test_exact_solution_residual_gpu():
+    inp = nasgen.make_class("BT", "A", A=0.0)
+    g = gpu_rhs(inp.u, inp.forcing, inp.dt, strict=False)
+    assert np.abs(g[1:-1, 1:-1, 1:-1]).max() < 1e-13
+
+
+def test_sp_native_layout_descriptor():
+    """`dim` with another stride order: SP's native u(i,j,k,m) = [m][k][j][i]."""
+    inp = nasgen.make_inputs(30, 22, 14, seed=4, dt=0.002)
+    nz, ny, nx, _ = inp.u.shape
+    sy = sr.pitch(nx)
+    d = sr.Dims(nx, ny, nz, sy, sy * ny * nz, sy * ny)
+
+    def to_sp(a):
+        t = torch.zeros((5, nz, ny, sy), dtype=torch.float64)
+        t[..., :nx] = torch.from_numpy(a).permute(3, 0, 1, 2)
+        return t.cuda().contiguous()
+
+    du, df = to_sp(inp.u), to_sp(inp.forcing)
+    dr = torch.full_like(du, float("nan"))
+    c = sr.coeffs_nas(nx, ny, nz, inp.dt)
+    sr.rhs(du, df, dr, nx, c, strict=True, dims=d)
+    torch.cuda.synchronize()
+    g = dr[..., :nx].permute(1, 2, 3, 0).cpu().numpy()
+    assert np.array_equal(g, oracle_rhs(inp))
+
+
+@pytest.mark.parametrize("nz,p", [(12, 2), (36, 3), (64, 2), (41, 4), (102, 8), (24, 8)])
+@pytest.mark.parametrize("split", [False, True])
+def test_slab_decomposition_bitwise(nz, p, split):
+    """z-slabs computed one after another on one GPU (ghost planes copied from
+    the global array) reproduce the single-GPU result bit for bit."""
+    nx, ny = 21, 18
+    inp = nasgen.make_inputs(nx, ny, nz, seed=5, dt=0.001)
+    c = sr.coeffs_nas(nx, ny, nz, inp.dt)
+    du, df = sr.pack(inp.u), sr.pack(inp.forcing)
+    ref = torch.full_like(du, float("nan"))
+    sr.rhs(du, df, ref, nx, c, strict=False)
+    out = torch.full_like(du, float("nan"))
+    base, rem = divmod(nz, p)
+    k0 = 0
+    for r in range(p):
+        nzl = base + (1 if r < rem else 0)
+        us = torch.zeros((nzl + 4,) + tuple(du.shape[1:]), dtype=torch.float64, device="cuda")
+        lo, hi = max(k0 - 2, 0), min(k0 + nzl + 2, nz)
+        us[lo - (k0 - 2):hi - (k0 - 2)] = du[lo:hi]
+        fs = df[k0:k0 + nzl].contiguous()
+        rs = torch.full_like(fs, float("nan"))
+        if split:
+            sr.rhs_slab(us, fs, rs, nx, nz, k0, c, part=sr.SAFARA_PART_INTERIOR)
+            sr.rhs_slab(us, fs, rs, nx, nz, k0, c, part=sr.SAFARA_PART_EDGE)
+        else:
+            sr.rhs_slab(us, fs, rs, nx, nz, k0, c, part=sr.SAFARA_PART_ALL)
+        out[k0:k0 + nzl] = rs
+        k0 += nzl
+    torch.cuda.synchronize()
+    a, b = sr.unpack(out, nx), sr.unpack(ref, nx)
+    assert np.array_equal(a, b)
+
+
+def test_host_e2e_path():
+    inp = nasgen.make_class("SP", "W", seed=6)
+    nz, ny, nx, _ = inp.u.shape
+    hu, hf = sr.pack(inp.u, pin=True), sr.pack(inp.forcing, pin=True)
+    hr = torch.zeros_like(hu).pin_memory()
+    du, df, dr = (torch.empty(hu.shape, dtype=torch.float64, device="cuda") for _ in range(3))
+    c = sr.coeffs_nas(nx, ny, nz, inp.dt)
+    sr.rhs_host(hu, hf, hr, du, df, dr, nx, c, strict=True)
+    torch.cuda.synchronize()
+    assert np.array_equal(sr.unpack(hr, nx), oracle_rhs(inp))
+
+
+def test_error_paths():
+    nx = ny = nz = 12
+    c = sr.coeffs_nas(nx, ny, nz, 0.01)
+    du = sr.empty_field(nx, ny, nz)
+    df = sr.empty_field(nx, ny, nz)
+    dr = sr.empty_field(nx, ny, nz)
+    with pytest.raises(sr.SafaraError) as e:      # rhs aliases u
+        sr.rhs(du, df, du, nx, c)
+    assert e.value.code == -1
+    flat = torch.empty(du.numel() + 1, dtype=torch.float64, device="cuda")
+    mis = flat[1:].view(du.shape)                 # 8-byte, not 16-byte, aligned
+    with pytest.raises(sr.SafaraError) as e:
+        sr.rhs(mis, df, dr, nx, c)
+    assert e.value.code == -4
+    small = sr.empty_field(5, 5, 5)
+    with pytest.raises(sr.SafaraError) as e:
+        sr.rhs(small, small.clone(), small.clone(), 5, c)
+    assert e.value.code == -2
+    # slab with a single owned plane
+    us = sr.empty_field(nx, ny, 5)
+    fs = sr.empty_field(nx, ny, 1)
+    with pytest.raises(sr.SafaraError) as e:
+        sr.rhs_slab(us, fs, fs.clone(), nx, nz, 3, c)
+    assert e.value.code == -2
+
+
+def test_kernel_info_zero_spill():
+    for strict in (False, True):
+        k = sr.kernel_info(strict)
+        assert k["local_bytes"] == 0
+        assert k["ctas_per_sm"] >= 1
+        assert k["regs_per_thread"] <= 255
