@@ -29,6 +29,8 @@
 //    c6).  Where NAS multiplies by 2.0 or 4.0 (exact scalings) the subtract
 //    is a single fma, which rounds identically.
 #pragma once
+#include <cstdio>
+
 #include "safara_internal.h"
 
 namespace safara {
@@ -254,8 +256,15 @@ __device__ __forceinline__ void issue_plane(const CUtensorMap *tmap, const Param
     const int c1 = P.pos_j == 1 ? jc : (P.pos_m == 1 ? 0 : kb);
     const int c2 = P.pos_j == 2 ? jc : (P.pos_m == 2 ? 0 : kb);
     const int c3 = P.pos_j == 3 ? jc : (P.pos_m == 3 ? 0 : kb);
+#ifdef SAFARA_DBG
+    if (blockIdx.x == 0)
+        printf("issue k=%d seq=%u slot=%d map=%p w0=%llx dst=%u bar=%u c=(%d,%d,%d,%d) pos=%d%d%d\n", k, seq, slot,
+               (const void *)tmap, (unsigned long long)reinterpret_cast<const uint64_t *>(tmap)[0],
+               smem_u32(su + (size_t)slot * U_SLOT), smem_u32(&mbar[slot]), i0 - HX, c1, c2, c3,
+               P.pos_j, P.pos_m, P.pos_k);
+#endif
     mbar_expect_tx(&mbar[slot], TMA_BYTES);
-    tma_load_4d(su + (size_t)slot * U_PLANE, tmap, &mbar[slot], i0 - 2, c1, c2, c3);
+    tma_load_4d(su + (size_t)slot * U_SLOT, tmap, &mbar[slot], i0 - HX, c1, c2, c3);
 }
 
 __device__ __forceinline__ void wait_plane(uint64_t *mbar, uint32_t seq) {
@@ -266,7 +275,7 @@ __device__ __forceinline__ void wait_plane(uint64_t *mbar, uint32_t seq) {
 __device__ __forceinline__ void rhs_body(const CUtensorMap *tmap, const Params &P) {
     extern __shared__ __align__(128) unsigned char smem_raw[];
     double *su = reinterpret_cast<double *>(smem_raw);
-    double2 *sa = reinterpret_cast<double2 *>(su + (size_t)STAGES * U_PLANE);
+    double2 *sa = reinterpret_cast<double2 *>(su + (size_t)STAGES * U_SLOT);
     uint64_t *mbar = reinterpret_cast<uint64_t *>(sa + (size_t)AUX_SLOTS * A_PLANE);
 
     const int tid = threadIdx.x;
@@ -320,7 +329,7 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *tmap, const Params &
         const bool mid_y = is_mid(j, P.ny);
         const Cases cx = cases_of(i, P.nx), cy = cases_of(j, P.ny);
 
-        const int uc = (ty + 2) * UX + (tx + 2);   // centre in the u tile
+        const int uc = (ty + 2) * UX + (tx + HX);  // centre in the u tile
         const int ac = (ty + 1) * AX + (tx + 1);   // centre in the aux tile
         const int ocol = i + P.sy * j;             // own column offset (dim)
 
@@ -340,7 +349,7 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *tmap, const Params &
         // plane ka: own column, own aux, ring aux
         wait_plane(mbar, seq0);
         {
-            const double *s = su + (size_t)((seq0) % STAGES) * U_PLANE;
+            const double *s = su + (size_t)((seq0) % STAGES) * U_SLOT;
             double2 *a = sa + (size_t)(ka % AUX_SLOTS) * A_PLANE;
             load5(w2, s, uc);
             if (in_grid) aux_of(w2[0], w2[1], w2[2], w2[3], r0, s0);
@@ -355,14 +364,14 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *tmap, const Params &
                 const int gi = i0 - 1 + ii, gj = j0 - 1 + jj;
                 double rr = 0.0, ss = 0.0;
                 if (gi >= 0 && gi < P.nx && gj >= 0 && gj < P.ny) {
-                    const int ui = (jj + 1) * UX + (ii + 1);
+                    const int ui = (jj + 1) * UX + (ii + HX - 1);
                     aux_of(s[ui], s[UPM + ui], s[2 * UPM + ui], s[3 * UPM + ui], rr, ss);
                 }
                 a[jj * AX + ii] = make_double2(rr, ss);
             }
         }
         wait_plane(mbar, seq0 + 1);
-        load5(w3, su + (size_t)((seq0 + 1) % STAGES) * U_PLANE, uc);
+        load5(w3, su + (size_t)((seq0 + 1) % STAGES) * U_SLOT, uc);
 
         for (int k = ka; k < kb; ++k) {
             const uint32_t sq_k = seq0 + (uint32_t)(k - ka);
@@ -376,7 +385,7 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *tmap, const Params &
             }
             // (1) own column u(k+2) into the window
             wait_plane(mbar, sq_k + 2);
-            load5(w4, su + (size_t)((sq_k + 2) % STAGES) * U_PLANE, uc);
+            load5(w4, su + (size_t)((sq_k + 2) % STAGES) * U_SLOT, uc);
             // (2) rho_i / square of plane k+1: own point (registers + smem) and halo ring
             {
                 if (in_grid) aux_of(w3[0], w3[1], w3[2], w3[3], rp1, sp1);
@@ -384,7 +393,7 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *tmap, const Params &
                 double2 *a = sa + (size_t)((k + 1) % AUX_SLOTS) * A_PLANE;
                 a[ac] = make_double2(rp1, sp1);
                 if (k + 1 < kb && tid < NRING) {
-                    const double *s = su + (size_t)((sq_k + 1) % STAGES) * U_PLANE;
+                    const double *s = su + (size_t)((sq_k + 1) % STAGES) * U_SLOT;
                     int ii, jj;
                     if (tid < AX) { ii = tid; jj = 0; }
                     else if (tid < 2 * AX) { ii = tid - AX; jj = AY - 1; }
@@ -393,7 +402,7 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *tmap, const Params &
                     const int gi = i0 - 1 + ii, gj = j0 - 1 + jj;
                     double rr = 0.0, ss = 0.0;
                     if (gi >= 0 && gi < P.nx && gj >= 0 && gj < P.ny) {
-                        const int ui = (jj + 1) * UX + (ii + 1);
+                        const int ui = (jj + 1) * UX + (ii + HX - 1);
                         aux_of(s[ui], s[UPM + ui], s[2 * UPM + ui], s[3 * UPM + ui], rr, ss);
                     }
                     a[jj * AX + ii] = make_double2(rr, ss);
@@ -407,7 +416,7 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *tmap, const Params &
             }
             // (5) the point (i, j, k)
             if (active) {
-                const double *s = su + (size_t)(sq_k % STAGES) * U_PLANE;
+                const double *s = su + (size_t)(sq_k % STAGES) * U_SLOT;
                 const double2 *a = sa + (size_t)(k % AUX_SLOTS) * A_PLANE;
 
                 double acc[5];

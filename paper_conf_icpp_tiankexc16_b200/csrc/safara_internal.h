@@ -17,17 +17,22 @@ constexpr int TX = 32;
 constexpr int TY = SAFARA_TY;
 constexpr int NTHREADS = TX * TY;
 constexpr int STAGES = 5;            // u planes in the TMA ring
-constexpr int UX = TX + 4;           // u tile incl. i halo of 2
+// u tile: i halo of 2 plus one pad column each side.  The TMA box's first
+// element must be 16-byte aligned (fp64: even i), and tiles start at odd i
+// (interior begins at i = 1), so the box starts at i0 - 3 and is TX + 6 wide.
+constexpr int HX = 3;                // u-tile column of the tile's first i
+constexpr int UX = TX + 2 * HX;
 constexpr int UY = TY + 4;           // u tile incl. j halo of 2
 constexpr int AX = TX + 2;           // aux (rho_i, square) tile incl. halo of 1
 constexpr int AY = TY + 2;
 constexpr int AUX_SLOTS = 3;         // aux planes k, k+1 (being written), k+2
-constexpr int U_PLANE = UX * UY * 5; // doubles per ring slot (one TMA box)
+constexpr int U_PLANE = UX * UY * 5; // doubles in one TMA box (one u plane tile)
+constexpr int U_SLOT = ((U_PLANE * 8 + 127) / 128) * 128 / 8;  // slot stride: TMA dst 128 B aligned
 constexpr int A_PLANE = AX * AY;     // double2 {rho_i, square} per aux slot
 constexpr int NRING = 2 * AX + 2 * TY;  // aux halo points recomputed per plane
 constexpr uint32_t TMA_BYTES = U_PLANE * 8u;
 constexpr size_t SMEM_BYTES =
-    (size_t)STAGES * U_PLANE * 8 + (size_t)AUX_SLOTS * A_PLANE * 16 + STAGES * 8;
+    (size_t)STAGES * U_SLOT * 8 + (size_t)AUX_SLOTS * A_PLANE * 16 + STAGES * 8;
 constexpr int MIN_PLANES_PER_CTA = 4;
 
 // Device-side coefficients: safara_coeffs_t plus the constant products that
