@@ -11,7 +11,8 @@ import re
 import threading
 
 PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(PKG, "libsafara_rhs.so")
+# SAFARA_LIB overrides the library path (A/B experiments with variant builds).
+LIB_PATH = os.environ.get("SAFARA_LIB") or os.path.join(PKG, "libsafara_rhs.so")
 HEADER = os.path.join(os.path.dirname(PKG), "include", "safara.h")
 
 SAFARA_OK = 0

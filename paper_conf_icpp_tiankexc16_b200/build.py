@@ -35,15 +35,17 @@ def _mtime(p):
     return os.path.getmtime(p) if os.path.exists(p) else 0.0
 
 
-def build(force: bool = False, verbose: bool = False, extra: list[str] | None = None) -> str:
-    """Compile (if stale) and return the path of libsafara_rhs.so."""
+def build(force: bool = False, verbose: bool = False, extra: list[str] | None = None,
+          out: str | None = None) -> str:
+    """Compile (if stale) and return the path of libsafara_rhs.so (or ``out``)."""
     os.makedirs(BUILD, exist_ok=True)
+    lib = out or LIB
     extra = list(extra or [])
     srcs = [os.path.join(CSRC, u) for u, _ in UNITS] + [os.path.join(CSRC, d) for d in DEPS]
     srcs.append(os.path.join(INCLUDE, "safara.h"))
     newest = max(_mtime(s) for s in srcs)
-    if not force and _mtime(LIB) >= newest and not extra:
-        return LIB
+    if not force and _mtime(lib) >= newest and not extra:
+        return lib
     objs = []
     ptxas_log = []
     for unit, flags in UNITS:
@@ -55,18 +57,18 @@ def build(force: bool = False, verbose: bool = False, extra: list[str] | None = 
             raise RuntimeError(f"nvcc failed for {unit}")
         ptxas_log.append(f"== {unit} {' '.join(flags)}\n{res.stdout}{res.stderr}")
         objs.append(obj)
-    tmp = LIB + f".tmp{os.getpid()}"
+    tmp = lib + f".tmp{os.getpid()}"
     cmd = [NVCC, *ARCH, "-shared", "-cudart", "static", "-o", tmp, *objs]
     res = subprocess.run(cmd, capture_output=True, text=True)
     if res.returncode != 0:
         sys.stderr.write(res.stdout + res.stderr)
         raise RuntimeError("nvcc link failed")
-    os.replace(tmp, LIB)
-    with open(os.path.join(BUILD, "ptxas.txt"), "w") as fh:
+    os.replace(tmp, lib)
+    with open(os.path.join(BUILD, "ptxas.txt") if out is None else out + ".ptxas.txt", "w") as fh:
         fh.write("\n".join(ptxas_log))
     if verbose:
         print("\n".join(ptxas_log))
-    return LIB
+    return lib
 
 
 if __name__ == "__main__":

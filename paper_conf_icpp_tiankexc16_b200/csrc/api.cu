@@ -11,6 +11,7 @@
 #include <algorithm>
 #include <atomic>
 #include <cstdint>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 
@@ -30,6 +31,20 @@ struct DeviceState {
 };
 
 DeviceState g_dev[kMaxDevices];
+
+// Tuning knobs, read once at init from the environment (defaults are the
+// measured best).  SAFARA_L2PROMO: TMA L2 promotion
+// 0=none 1=64B 2=128B 3=256B.  SAFARA_CHUNK: planes per chunk of the
+// chunk-major work order (0 = whole column).
+struct Tune {
+    int l2promo = 0;
+    int chunk = 0;
+} g_tune;
+
+int env_int(const char *name, int dflt) {
+    const char *v = std::getenv(name);
+    return v && *v ? std::atoi(v) : dflt;
+}
 std::mutex g_mutex;
 PFN_cuTensorMapEncodeTiled_v12000 g_encode = nullptr;
 std::atomic<int64_t> g_launches{0};
@@ -119,9 +134,12 @@ int encode_u_map(CUtensorMap *map, const double *u, const safara_dims_t &d, int 
         if (ax[t].which == 1) *pos_m = t + 1;
         if (ax[t].which == 2) *pos_k = t + 1;
     }
+    const CUtensorMapL2promotion promo[4] = {
+        CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_64B,
+        CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B};
     CUresult r = g_encode(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 4, const_cast<double *>(u), gdim,
                           gstride, box, estride, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                          CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                          CU_TENSOR_MAP_SWIZZLE_NONE, promo[g_tune.l2promo & 3],
                           CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     return r == CUDA_SUCCESS ? SAFARA_OK : SAFARA_ERR_CUDA;
 }
@@ -150,7 +168,9 @@ int launch(const double *u, const double *f, double *r, const safara_dims_t &d, 
     p.nplanes = p.n0 + (p.kb1 - p.ka1);
     p.ntx = (d.nx - 2 + TX - 1) / TX;
     p.nty = (d.ny - 2 + TY - 1) / TY;
-    p.units = (long long)p.ntx * p.nty * p.nplanes;
+    p.ncol = p.ntx * p.nty;
+    p.units = (long long)p.ncol * p.nplanes;
+    p.chunk = std::max(1, std::min(g_tune.chunk > 0 ? g_tune.chunk : p.nplanes, p.nplanes));
     p.fk_lo = fk_lo; p.fk_hi = fk_hi;
     p.u = u; p.f = f; p.r = r;
     to_coef(*coeffs, p.c);
@@ -226,6 +246,8 @@ int safara_rhs_init(int device) {
     if (cudaGetDeviceCount(&count) != cudaSuccess || count < 1) return SAFARA_ERR_NO_DEVICE;
     if (device < 0 || device >= count || device >= kMaxDevices) return SAFARA_ERR_NO_DEVICE;
     if (g_dev[device].ready) return SAFARA_OK;
+    g_tune.l2promo = env_int("SAFARA_L2PROMO", g_tune.l2promo);
+    g_tune.chunk = env_int("SAFARA_CHUNK", g_tune.chunk);
     int major = 0, minor = 0, sms = 0;
     if (cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, device) ||
         cudaDeviceGetAttribute(&minor, cudaDevAttrComputeCapabilityMinor, device) ||

@@ -33,6 +33,10 @@
 
 #include "safara_internal.h"
 
+#ifndef SAFARA_FPREFETCH
+#define SAFARA_FPREFETCH 0
+#endif
+
 namespace safara {
 namespace dev {
 
@@ -248,7 +252,7 @@ __device__ __forceinline__ void copy_faces(const Params &P) {
 }
 
 __device__ __forceinline__ void issue_plane(const CUtensorMap *tmap, const Params &P,
-                                            double *su, uint64_t *mbar, int i0, int j0, int k,
+                                            double *su, uint64_t *full, int i0, int j0, int k,
                                             uint32_t seq) {
     const int slot = (int)(seq % STAGES);
     const int kb = k - P.k0 + P.ukoff;
@@ -256,35 +260,51 @@ __device__ __forceinline__ void issue_plane(const CUtensorMap *tmap, const Param
     const int c1 = P.pos_j == 1 ? jc : (P.pos_m == 1 ? 0 : kb);
     const int c2 = P.pos_j == 2 ? jc : (P.pos_m == 2 ? 0 : kb);
     const int c3 = P.pos_j == 3 ? jc : (P.pos_m == 3 ? 0 : kb);
-#ifdef SAFARA_DBG
-    if (blockIdx.x == 0)
-        printf("issue k=%d seq=%u slot=%d map=%p w0=%llx dst=%u bar=%u c=(%d,%d,%d,%d) pos=%d%d%d\n", k, seq, slot,
-               (const void *)tmap, (unsigned long long)reinterpret_cast<const uint64_t *>(tmap)[0],
-               smem_u32(su + (size_t)slot * U_SLOT), smem_u32(&mbar[slot]), i0 - HX, c1, c2, c3,
-               P.pos_j, P.pos_m, P.pos_k);
-#endif
-    mbar_expect_tx(&mbar[slot], TMA_BYTES);
-    tma_load_4d(su + (size_t)slot * U_SLOT, tmap, &mbar[slot], i0 - HX, c1, c2, c3);
+    mbar_expect_tx(&full[slot], TMA_BYTES);
+    tma_load_4d(su + (size_t)slot * U_SLOT, tmap, &full[slot], i0 - HX, c1, c2, c3);
 }
 
-__device__ __forceinline__ void wait_plane(uint64_t *mbar, uint32_t seq) {
-    mbar_wait(&mbar[seq % STAGES], (seq / STAGES) & 1u);
+__device__ __forceinline__ void wait_plane(uint64_t *full, uint32_t seq) {
+    mbar_wait(&full[seq % STAGES], (seq / STAGES) & 1u);
+}
+
+// Decode linear column-plane unit L (chunk-major: all column tiles advance
+// through the same band of k-planes together, so a plane's i/j halo that a
+// neighbouring tile fetched is still in L2) into (column, plane index) and the
+// number of units left in this (chunk, column) run.
+__device__ __forceinline__ void decode_unit(const Params &P, long long L, int &col, int &pidx,
+                                            int &run) {
+    const long long per_chunk = (long long)P.chunk * P.ncol;
+    const int c = (int)(L / per_chunk);
+    const long long rem = L - (long long)c * per_chunk;
+    const int kc = min(P.chunk, P.nplanes - c * P.chunk);
+    col = (int)(rem / kc);
+    const int off = (int)(rem - (long long)col * kc);
+    pidx = c * P.chunk + off;
+    run = kc - off;
 }
 
 // One CTA processes the column-plane units [blockIdx*units/ncta, ...).
+// Warps are decoupled: warp w owns row j0+w of the tile and never waits for
+// another warp except through the TMA ring (a slot is refilled by the last
+// warp to release it).
 __device__ __forceinline__ void rhs_body(const CUtensorMap *tmap, const Params &P) {
     extern __shared__ __align__(128) unsigned char smem_raw[];
     double *su = reinterpret_cast<double *>(smem_raw);
-    double2 *sa = reinterpret_cast<double2 *>(su + (size_t)STAGES * U_SLOT);
-    uint64_t *mbar = reinterpret_cast<uint64_t *>(sa + (size_t)AUX_SLOTS * A_PLANE);
+    uint64_t *full = reinterpret_cast<uint64_t *>(su + (size_t)STAGES * U_SLOT);
+    unsigned int *released = reinterpret_cast<unsigned int *>(full + STAGES);
 
     const int tid = threadIdx.x;
-    const int tx = tid % TX, ty = tid / TX;
+    const int tx = tid % TX, ty = tid / TX;  // lane = tx, warp = ty
+    const unsigned FULL = 0xffffffffu;
     const Coef &C = P.c;
 
     if (tid == 0) {
         prefetch_tmap(tmap);
-        for (int s = 0; s < STAGES; ++s) mbar_init(&mbar[s], 1);
+        for (int s = 0; s < STAGES; ++s) {
+            mbar_init(&full[s], 1);
+            released[s] = 0;
+        }
         fence_mbar_init();
     }
     __syncthreads();
@@ -297,11 +317,11 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *tmap, const Params &
 
     while (ub < ue) {
         // ---- segment: one column tile, a contiguous run of planes ----
-        const int col = (int)(ub / P.nplanes);
-        const int pidx = (int)(ub % P.nplanes);
+        int col, pidx, run;
+        decode_unit(P, ub, col, pidx, run);
         int ka, kb;
         {
-            const long long left = ue - ub;
+            const long long left = min((long long)run, ue - ub);
             if (pidx < P.n0) {
                 ka = P.ka0 + pidx;
                 kb = (int)min((long long)P.kb0, ka + left);
@@ -321,7 +341,7 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *tmap, const Params &
 
         if (tid == 0) {
             const int npre = nload < STAGES ? nload : STAGES;
-            for (int s = 0; s < npre; ++s) issue_plane(tmap, P, su, mbar, i0, j0, ka + s, seq0 + s);
+            for (int s = 0; s < npre; ++s) issue_plane(tmap, P, su, full, i0, j0, ka + s, seq0 + s);
         }
 
         // Case flags (global indices, reading c12).
@@ -330,7 +350,6 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *tmap, const Params &
         const Cases cx = cases_of(i, P.nx), cy = cases_of(j, P.ny);
 
         const int uc = (ty + 2) * UX + (tx + HX);  // centre in the u tile
-        const int ac = (ty + 1) * AX + (tx + 1);   // centre in the aux tile
         const int ocol = i + P.sy * j;             // own column offset (dim)
 
         // Register window u(:, k-2..k+2) and own rho_i/square at k-1..k+1.
@@ -346,78 +365,56 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *tmap, const Params &
             if (in_grid && kbm1 >= 0) aux_of(w1[0], w1[1], w1[2], w1[3], rm1, sm1);
             else { rm1 = 0.0; sm1 = 0.0; }
         }
-        // plane ka: own column, own aux, ring aux
-        wait_plane(mbar, seq0);
-        {
-            const double *s = su + (size_t)((seq0) % STAGES) * U_SLOT;
-            double2 *a = sa + (size_t)(ka % AUX_SLOTS) * A_PLANE;
-            load5(w2, s, uc);
-            if (in_grid) aux_of(w2[0], w2[1], w2[2], w2[3], r0, s0);
-            else { r0 = 0.0; s0 = 0.0; }
-            a[ac] = make_double2(r0, s0);
-            if (tid < NRING) {
-                int ii, jj;
-                if (tid < AX) { ii = tid; jj = 0; }
-                else if (tid < 2 * AX) { ii = tid - AX; jj = AY - 1; }
-                else if (tid < 2 * AX + TY) { ii = 0; jj = 1 + tid - 2 * AX; }
-                else { ii = AX - 1; jj = 1 + tid - 2 * AX - TY; }
-                const int gi = i0 - 1 + ii, gj = j0 - 1 + jj;
-                double rr = 0.0, ss = 0.0;
-                if (gi >= 0 && gi < P.nx && gj >= 0 && gj < P.ny) {
-                    const int ui = (jj + 1) * UX + (ii + HX - 1);
-                    aux_of(s[ui], s[UPM + ui], s[2 * UPM + ui], s[3 * UPM + ui], rr, ss);
-                }
-                a[jj * AX + ii] = make_double2(rr, ss);
-            }
-        }
-        wait_plane(mbar, seq0 + 1);
+        wait_plane(full, seq0);
+        load5(w2, su + (size_t)(seq0 % STAGES) * U_SLOT, uc);
+        if (in_grid) aux_of(w2[0], w2[1], w2[2], w2[3], r0, s0);
+        else { r0 = 0.0; s0 = 0.0; }
+        wait_plane(full, seq0 + 1);
         load5(w3, su + (size_t)((seq0 + 1) % STAGES) * U_SLOT, uc);
+
+#if SAFARA_FPREFETCH
+        double fn[5];
+        {
+            const int kl = ka - P.k0;
+#pragma unroll
+            for (int m = 0; m < 5; ++m)
+                fn[m] = active ? __ldcs(P.f + ocol + P.sm * m + P.sk * kl) : 0.0;
+        }
+#endif
 
         for (int k = ka; k < kb; ++k) {
             const uint32_t sq_k = seq0 + (uint32_t)(k - ka);
-            // (0) stream forcing(k): used once, never staged (reuse count 1)
+            // forcing is used once (reuse count 1): streamed, never staged.
             double fr[5];
+#if SAFARA_FPREFETCH
+            // prefetched one step ahead; stream forcing(k+1)
+#pragma unroll
+            for (int m = 0; m < 5; ++m) fr[m] = fn[m];
+            {
+                const int kl = k + 1 - P.k0;
+                const bool ok = active && (k + 1 < kb);
+#pragma unroll
+                for (int m = 0; m < 5; ++m)
+                    fn[m] = ok ? __ldcs(P.f + ocol + P.sm * m + P.sk * kl) : 0.0;
+            }
+#else
             {
                 const int kl = k - P.k0;
 #pragma unroll
                 for (int m = 0; m < 5; ++m)
                     fr[m] = active ? __ldcs(P.f + ocol + P.sm * m + P.sk * kl) : 0.0;
             }
-            // (1) own column u(k+2) into the window
-            wait_plane(mbar, sq_k + 2);
+#endif
+            // own column u(k+2) into the window; own rho_i/square of plane k+1
+            wait_plane(full, sq_k + 2);
             load5(w4, su + (size_t)((sq_k + 2) % STAGES) * U_SLOT, uc);
-            // (2) rho_i / square of plane k+1: own point (registers + smem) and halo ring
+            if (in_grid) aux_of(w3[0], w3[1], w3[2], w3[3], rp1, sp1);
+            else { rp1 = 0.0; sp1 = 0.0; }
+
+            // ---- the point (i, j, k): every lane runs it (shuffles), only
+            // active lanes store ----
             {
-                if (in_grid) aux_of(w3[0], w3[1], w3[2], w3[3], rp1, sp1);
-                else { rp1 = 0.0; sp1 = 0.0; }
-                double2 *a = sa + (size_t)((k + 1) % AUX_SLOTS) * A_PLANE;
-                a[ac] = make_double2(rp1, sp1);
-                if (k + 1 < kb && tid < NRING) {
-                    const double *s = su + (size_t)((sq_k + 1) % STAGES) * U_SLOT;
-                    int ii, jj;
-                    if (tid < AX) { ii = tid; jj = 0; }
-                    else if (tid < 2 * AX) { ii = tid - AX; jj = AY - 1; }
-                    else if (tid < 2 * AX + TY) { ii = 0; jj = 1 + tid - 2 * AX; }
-                    else { ii = AX - 1; jj = 1 + tid - 2 * AX - TY; }
-                    const int gi = i0 - 1 + ii, gj = j0 - 1 + jj;
-                    double rr = 0.0, ss = 0.0;
-                    if (gi >= 0 && gi < P.nx && gj >= 0 && gj < P.ny) {
-                        const int ui = (jj + 1) * UX + (ii + HX - 1);
-                        aux_of(s[ui], s[UPM + ui], s[2 * UPM + ui], s[3 * UPM + ui], rr, ss);
-                    }
-                    a[jj * AX + ii] = make_double2(rr, ss);
-                }
-            }
-            __syncthreads();
-            // (3) refill the slot plane k-1 used (every thread is past step k-1)
-            if (tid == 0 && k > ka) {
-                const int kn = k - 1 + STAGES;
-                if (kn <= kb + 1) issue_plane(tmap, P, su, mbar, i0, j0, kn, sq_k - 1 + STAGES);
-            }
-            // (5) the point (i, j, k)
-            if (active) {
                 const double *s = su + (size_t)(sq_k % STAGES) * U_SLOT;
-                const double2 *a = sa + (size_t)(k % AUX_SLOTS) * A_PLANE;
 
                 double acc[5];
 #pragma unroll
@@ -433,10 +430,24 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *tmap, const Params &
 #pragma unroll
                 for (int m = 0; m < 5; ++m) six[m] = 6.0 * w2[m];
 
-                // xi
+                // xi: rho_i/square of i+-1 are the neighbour lanes' own values;
+                // lanes 0 and 31 evaluate their outside neighbour themselves.
                 {
-                    const Nb p = load_nb(s, a, uc + 1, ac + 1);
-                    const Nb q = load_nb(s, a, uc - 1, ac - 1);
+                    Nb p, q;
+                    load5(p.u, s, uc + 1);
+                    load5(q.u, s, uc - 1);
+                    p.rho = __shfl_down_sync(FULL, r0, 1);
+                    p.sq = __shfl_down_sync(FULL, s0, 1);
+                    q.rho = __shfl_up_sync(FULL, r0, 1);
+                    q.sq = __shfl_up_sync(FULL, s0, 1);
+                    {
+                        const bool left = (tx == 0);
+                        double re, se;
+                        aux_of(left ? q.u[0] : p.u[0], left ? q.u[1] : p.u[1],
+                               left ? q.u[2] : p.u[2], left ? q.u[3] : p.u[3], re, se);
+                        if (left) { q.rho = re; q.sq = se; }
+                        if (tx == TX - 1) { p.rho = re; p.sq = se; }
+                    }
                     flux_dir<1>(acc, w2, vc, qsc, pc, p, q, C, 0);
                     double pp[5], qq[5];
                     load5(pp, s, uc + 2);
@@ -444,10 +455,14 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *tmap, const Params &
                     if (mid_x) diss_dir<false>(acc, qq, q.u, w2, six, p.u, pp, C.dssp, cx);
                     else diss_dir<true>(acc, qq, q.u, w2, six, p.u, pp, C.dssp, cx);
                 }
-                // eta
+                // eta: rows j+-1 belong to other warps; evaluate their
+                // rho_i/square from the u values loaded for the stencil.
                 {
-                    const Nb p = load_nb(s, a, uc + UX, ac + AX);
-                    const Nb q = load_nb(s, a, uc - UX, ac - AX);
+                    Nb p, q;
+                    load5(p.u, s, uc + UX);
+                    load5(q.u, s, uc - UX);
+                    aux_of(p.u[0], p.u[1], p.u[2], p.u[3], p.rho, p.sq);
+                    aux_of(q.u[0], q.u[1], q.u[2], q.u[3], q.rho, q.sq);
                     flux_dir<2>(acc, w2, vc, qsc, pc, p, q, C, 1);
                     double pp[5], qq[5];
                     load5(pp, s, uc + 2 * UX);
@@ -469,11 +484,26 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *tmap, const Params &
                     if (is_mid(k, P.nz)) diss_dir<false>(acc, w0, w1, w2, six, w3, w4, C.dssp, Cases{});
                     else diss_dir<true>(acc, w0, w1, w2, six, w3, w4, C.dssp, cases_of(k, P.nz));
                 }
-                const int o = ocol + P.sk * (k - P.k0);
+                if (active) {
+                    const int o = ocol + P.sk * (k - P.k0);
 #pragma unroll
-                for (int m = 0; m < 5; ++m) __stcs(P.r + o + P.sm * m, acc[m] * C.dt);
+                    for (int m = 0; m < 5; ++m) __stcs(P.r + o + P.sm * m, acc[m] * C.dt);
+                }
             }
-            // (6) rotate the windows
+            // release plane k's slot; the last warp out refills it with k+STAGES
+            __syncwarp();
+            if (tx == 0) {
+                const int slot = (int)(sq_k % STAGES);
+                __threadfence_block();
+                const unsigned old = atomicAdd(&released[slot], 1u);
+                if (old == (unsigned)(TY - 1)) {
+                    released[slot] = 0;
+                    __threadfence_block();
+                    const int kn = k + STAGES;
+                    if (kn <= kb + 1) issue_plane(tmap, P, su, full, i0, j0, kn, sq_k + STAGES);
+                }
+            }
+            // rotate the windows
 #pragma unroll
             for (int m = 0; m < 5; ++m) {
                 w0[m] = w1[m];
@@ -485,7 +515,11 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *tmap, const Params &
             r0 = rp1; s0 = sp1;
         }
         seq0 += (uint32_t)nload;
-        __syncthreads();  // every slot / aux plane of this segment is consumed
+        // Segment end: every warp has consumed every plane; planes kb, kb+1
+        // were never released, so clear the counters before the next segment.
+        __syncthreads();
+        if (tid < STAGES) released[tid] = 0;
+        __syncthreads();
     }
 }
 

@@ -12,7 +12,7 @@ namespace safara {
 // CTA tile: TX x TY (i, j) columns, one thread per column marching along k.
 constexpr int TX = 32;
 #ifndef SAFARA_TY
-#define SAFARA_TY 10
+#define SAFARA_TY 12
 #endif
 constexpr int TY = SAFARA_TY;
 constexpr int NTHREADS = TX * TY;
@@ -23,16 +23,10 @@ constexpr int STAGES = 5;            // u planes in the TMA ring
 constexpr int HX = 3;                // u-tile column of the tile's first i
 constexpr int UX = TX + 2 * HX;
 constexpr int UY = TY + 4;           // u tile incl. j halo of 2
-constexpr int AX = TX + 2;           // aux (rho_i, square) tile incl. halo of 1
-constexpr int AY = TY + 2;
-constexpr int AUX_SLOTS = 3;         // aux planes k, k+1 (being written), k+2
 constexpr int U_PLANE = UX * UY * 5; // doubles in one TMA box (one u plane tile)
 constexpr int U_SLOT = ((U_PLANE * 8 + 127) / 128) * 128 / 8;  // slot stride: TMA dst 128 B aligned
-constexpr int A_PLANE = AX * AY;     // double2 {rho_i, square} per aux slot
-constexpr int NRING = 2 * AX + 2 * TY;  // aux halo points recomputed per plane
 constexpr uint32_t TMA_BYTES = U_PLANE * 8u;
-constexpr size_t SMEM_BYTES =
-    (size_t)STAGES * U_SLOT * 8 + (size_t)AUX_SLOTS * A_PLANE * 16 + STAGES * 8;
+constexpr size_t SMEM_BYTES = (size_t)STAGES * U_SLOT * 8 + STAGES * 8 + STAGES * 4;
 constexpr int MIN_PLANES_PER_CTA = 4;
 
 // Device-side coefficients: safara_coeffs_t plus the constant products that
@@ -53,6 +47,8 @@ struct Params {
     int ka0, kb0, ka1, kb1;// global planes to compute: [ka0,kb0) U [ka1,kb1)
     int n0, nplanes;       // n0 = kb0-ka0, nplanes = n0 + (kb1-ka1)
     int ntx, nty;          // column tiles
+    int ncol;              // ntx * nty
+    int chunk;             // planes per chunk of the chunk-major unit order
     int ncta;              // CTAs in the grid
     long long units;       // ntx*nty*nplanes (column-plane work items)
     int fk_lo, fk_hi;      // local planes whose boundary faces this launch copies
