@@ -35,10 +35,12 @@ DeviceState g_dev[kMaxDevices];
 // Tuning knobs, read once at init from the environment (defaults are the
 // measured best).  SAFARA_L2PROMO: TMA L2 promotion
 // 0=none 1=64B 2=128B 3=256B.  SAFARA_CHUNK: planes per chunk of the
-// chunk-major work order (0 = whole column).
+// chunk-major work order (0 = whole column).  SAFARA_SCHED: 0 = balanced
+// contiguous ranges, 1 = lockstep (column tile, k-part) per CTA.
 struct Tune {
     int l2promo = 0;
     int chunk = 0;
+    int sched = 1;  // 0 = balanced contiguous ranges, 1 = lockstep (column, k-part)
 } g_tune;
 
 int env_int(const char *name, int dflt) {
@@ -116,15 +118,16 @@ void to_coef(const safara_coeffs_t &in, Coef &c) {
     }
 }
 
-// 4-D tensor map over u: dim0 = i, then (j, m, k) ordered by stride.
-int encode_u_map(CUtensorMap *map, const double *u, const safara_dims_t &d, int nzb, int *pos_j,
-                 int *pos_m, int *pos_k) {
+// 4-D tensor map over a field: dim0 = i, then (j, m, k) ordered by stride;
+// box (box_x, box_y, 5, 1), so the smem tile is [m][j][i] for any stride order.
+int encode_map(CUtensorMap *map, const double *base, const safara_dims_t &d, int nplanes,
+               int box_x, int box_y, int *pos_j, int *pos_m, int *pos_k) {
     struct Ax { int which; long long stride, extent, box; } ax[3] = {
-        {0, d.sy, d.ny, UY}, {1, d.sm, 5, 5}, {2, d.sk, nzb, 1}};
+        {0, d.sy, d.ny, box_y}, {1, d.sm, 5, 5}, {2, d.sk, nplanes, 1}};
     std::sort(ax, ax + 3, [](const Ax &a, const Ax &b) { return a.stride < b.stride; });
     cuuint64_t gdim[4] = {(cuuint64_t)d.nx, 0, 0, 0};
     cuuint64_t gstride[3];
-    cuuint32_t box[4] = {(cuuint32_t)UX, 0, 0, 0};
+    cuuint32_t box[4] = {(cuuint32_t)box_x, 0, 0, 0};
     cuuint32_t estride[4] = {1, 1, 1, 1};
     for (int t = 0; t < 3; ++t) {
         gdim[t + 1] = (cuuint64_t)ax[t].extent;
@@ -137,7 +140,7 @@ int encode_u_map(CUtensorMap *map, const double *u, const safara_dims_t &d, int 
     const CUtensorMapL2promotion promo[4] = {
         CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_64B,
         CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B};
-    CUresult r = g_encode(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 4, const_cast<double *>(u), gdim,
+    CUresult r = g_encode(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 4, const_cast<double *>(base), gdim,
                           gstride, box, estride, CU_TENSOR_MAP_INTERLEAVE_NONE,
                           CU_TENSOR_MAP_SWIZZLE_NONE, promo[g_tune.l2promo & 3],
                           CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
@@ -147,7 +150,8 @@ int encode_u_map(CUtensorMap *map, const double *u, const safara_dims_t &d, int 
 // Shared launch path.  u has nzu planes, u plane = k - k0 + ukoff; forcing
 // and rhs start at global plane k0.  [ka0,kb0) U [ka1,kb1) are computed;
 // boundary faces of local planes [fk_lo, fk_hi) are copied.
-int launch(const double *u, const double *f, double *r, const safara_dims_t &d, int nzu, int k0,
+int launch(const double *u, const double *f, double *r, const safara_dims_t &d, int nzu, int nzf,
+           int k0,
            int ukoff, int ka0, int kb0, int ka1, int kb1, int fk_lo, int fk_hi,
            const safara_coeffs_t *coeffs, int flags, cudaStream_t stream) {
     int dev;
@@ -169,7 +173,9 @@ int launch(const double *u, const double *f, double *r, const safara_dims_t &d, 
     p.ntx = (d.nx - 2 + TX - 1) / TX;
     p.nty = (d.ny - 2 + TY - 1) / TY;
     p.ncol = p.ntx * p.nty;
-    p.units = (long long)p.ncol * p.nplanes;
+    const long long units = (long long)p.ncol * p.nplanes;
+    if (units >= (1LL << 31)) return SAFARA_ERR_TOO_LARGE;
+    p.units = (int)units;
     p.chunk = std::max(1, std::min(g_tune.chunk > 0 ? g_tune.chunk : p.nplanes, p.nplanes));
     p.fk_lo = fk_lo; p.fk_hi = fk_hi;
     p.u = u; p.f = f; p.r = r;
@@ -178,18 +184,32 @@ int launch(const double *u, const double *f, double *r, const safara_dims_t &d, 
     const bool strict = (flags & SAFARA_FLAG_STRICT) != 0;
     const int per_sm = strict ? st.ctas_strict : st.ctas_fast;
     const long long max_ctas = (long long)std::max(per_sm, 1) * st.sms;
-    long long ncta = (p.units + MIN_PLANES_PER_CTA - 1) / MIN_PLANES_PER_CTA;
-    ncta = std::min(ncta, max_ctas);
+    long long ncta;
+    if (g_tune.sched == 1 && p.ncol <= max_ctas && p.nplanes > 0) {
+        // Lockstep: every CTA owns one (column tile, k-part) and all parts
+        // start together, so neighbouring tiles read a plane's shared halo
+        // at the same time and the second read hits L2.
+        long long parts = max_ctas / p.ncol;
+        parts = std::min<long long>(parts, std::max(1, p.nplanes / MIN_PLANES_PER_CTA));
+        ncta = p.ncol * std::max<long long>(parts, 1);
+    } else {
+        ncta = (p.units + MIN_PLANES_PER_CTA - 1) / MIN_PLANES_PER_CTA;
+        ncta = std::min(ncta, max_ctas);
+    }
     if (ncta < 1) {
         if (fk_hi <= fk_lo) return SAFARA_OK;  // nothing to do
         ncta = std::min<long long>(max_ctas, 16);
     }
     p.ncta = (int)ncta;
 
-    CUtensorMap map;
-    rc = encode_u_map(&map, u, d, nzu, &p.pos_j, &p.pos_m, &p.pos_k);
+    CUtensorMap umap, fmap;
+    int pj, pm, pk;
+    rc = encode_map(&umap, u, d, nzu, UX, UY, &p.pos_j, &p.pos_m, &p.pos_k);
     if (rc) return rc;
-    cudaError_t e = strict ? launch_rhs_strict(map, p, stream) : launch_rhs_fast(map, p, stream);
+    rc = encode_map(&fmap, f, d, nzf, FX, TY, &pj, &pm, &pk);
+    if (rc) return rc;
+    cudaError_t e = strict ? launch_rhs_strict(umap, fmap, p, stream)
+                           : launch_rhs_fast(umap, fmap, p, stream);
     if (e != cudaSuccess) return SAFARA_ERR_CUDA;
     g_launches.fetch_add(1, std::memory_order_relaxed);
     return SAFARA_OK;
@@ -248,6 +268,7 @@ int safara_rhs_init(int device) {
     if (g_dev[device].ready) return SAFARA_OK;
     g_tune.l2promo = env_int("SAFARA_L2PROMO", g_tune.l2promo);
     g_tune.chunk = env_int("SAFARA_CHUNK", g_tune.chunk);
+    g_tune.sched = env_int("SAFARA_SCHED", g_tune.sched);
     int major = 0, minor = 0, sms = 0;
     if (cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, device) ||
         cudaDeviceGetAttribute(&minor, cudaDevAttrComputeCapabilityMinor, device) ||
@@ -299,7 +320,7 @@ int safara_rhs_ex(const double *u, const double *forcing, double *rhs, const saf
     rc = check_ptrs(u, bytes, forcing, bytes, rhs, bytes);
     if (rc) return rc;
     const int nz = dims->nz;
-    return launch(u, forcing, rhs, *dims, nz, 0, 0, 1, nz - 1, 0, 0, 0, nz, coeffs, flags,
+    return launch(u, forcing, rhs, *dims, nz, nz, 0, 0, 1, nz - 1, 0, 0, 0, nz, coeffs, flags,
                   (cudaStream_t)stream);
 }
 
@@ -335,7 +356,7 @@ int safara_rhs_slab(const double *u_slab, const double *forcing_slab, double *rh
         ka0 = lo; kb0 = e0; ka1 = e1; kb1 = hi;
         fk_lo = fk_hi = 0;
     }
-    return launch(u_slab, forcing_slab, rhs_slab, *dims, nzu, k0, 2, ka0, kb0, ka1, kb1, fk_lo,
+    return launch(u_slab, forcing_slab, rhs_slab, *dims, nzu, nzl, k0, 2, ka0, kb0, ka1, kb1, fk_lo,
                   fk_hi, coeffs, flags, (cudaStream_t)stream);
 }
 

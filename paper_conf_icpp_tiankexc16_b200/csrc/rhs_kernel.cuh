@@ -33,9 +33,6 @@
 
 #include "safara_internal.h"
 
-#ifndef SAFARA_FPREFETCH
-#define SAFARA_FPREFETCH 0
-#endif
 
 namespace safara {
 namespace dev {
@@ -251,17 +248,27 @@ __device__ __forceinline__ void copy_faces(const Params &P) {
     }
 }
 
-__device__ __forceinline__ void issue_plane(const CUtensorMap *tmap, const Params &P,
-                                            double *su, uint64_t *full, int i0, int j0, int k,
-                                            uint32_t seq) {
+// Stage plane k: the u tile (halo 2 in i/j) and, for planes that are
+// computed, the forcing tile, both onto the slot's mbarrier.
+__device__ __forceinline__ void issue_plane(const CUtensorMap *umap, const CUtensorMap *fmap,
+                                            const Params &P, double *su, uint64_t *full, int i0,
+                                            int j0, int k, bool with_f, uint32_t seq) {
     const int slot = (int)(seq % STAGES);
     const int kb = k - P.k0 + P.ukoff;
+    const int kf = k - P.k0;
     const int jc = j0 - 2;
     const int c1 = P.pos_j == 1 ? jc : (P.pos_m == 1 ? 0 : kb);
     const int c2 = P.pos_j == 2 ? jc : (P.pos_m == 2 ? 0 : kb);
     const int c3 = P.pos_j == 3 ? jc : (P.pos_m == 3 ? 0 : kb);
-    mbar_expect_tx(&full[slot], TMA_BYTES);
-    tma_load_4d(su + (size_t)slot * U_SLOT, tmap, &full[slot], i0 - HX, c1, c2, c3);
+    double *dst = su + (size_t)slot * SLOT;
+    mbar_expect_tx(&full[slot], with_f ? TMA_BYTES + TMA_BYTES_F : TMA_BYTES);
+    tma_load_4d(dst, umap, &full[slot], i0 - HX, c1, c2, c3);
+    if (with_f) {
+        const int f1 = P.pos_j == 1 ? j0 : (P.pos_m == 1 ? 0 : kf);
+        const int f2 = P.pos_j == 2 ? j0 : (P.pos_m == 2 ? 0 : kf);
+        const int f3 = P.pos_j == 3 ? j0 : (P.pos_m == 3 ? 0 : kf);
+        tma_load_4d(dst + U_SLOT, fmap, &full[slot], i0 - 1, f1, f2, f3);
+    }
 }
 
 __device__ __forceinline__ void wait_plane(uint64_t *full, uint32_t seq) {
@@ -272,35 +279,175 @@ __device__ __forceinline__ void wait_plane(uint64_t *full, uint32_t seq) {
 // through the same band of k-planes together, so a plane's i/j halo that a
 // neighbouring tile fetched is still in L2) into (column, plane index) and the
 // number of units left in this (chunk, column) run.
-__device__ __forceinline__ void decode_unit(const Params &P, long long L, int &col, int &pidx,
+// floor(c * units / ncta) without a 64-bit division subroutine call (keeps
+// the loop control visibly warp-uniform, so shuffles need no collective path)
+__device__ __forceinline__ int split_point(int c, int units, int ncta) {
+    const long long num = (long long)c * units;
+    long long q = (long long)((double)num / (double)ncta);
+    while (q * ncta > num) --q;
+    while ((q + 1) * ncta <= num) ++q;
+    return (int)q;
+}
+
+__device__ __forceinline__ void decode_unit(const Params &P, int L, int &col, int &pidx,
                                             int &run) {
-    const long long per_chunk = (long long)P.chunk * P.ncol;
-    const int c = (int)(L / per_chunk);
-    const long long rem = L - (long long)c * per_chunk;
+    const int per_chunk = P.chunk * P.ncol;
+    const int c = L / per_chunk;
+    const int rem = L - c * per_chunk;
     const int kc = min(P.chunk, P.nplanes - c * P.chunk);
-    col = (int)(rem / kc);
-    const int off = (int)(rem - (long long)col * kc);
+    col = rem / kc;
+    const int off = rem - col * kc;
     pidx = c * P.chunk + off;
     run = kc - off;
+}
+
+// Per-segment state of one thread.  The register window is a 5-entry ring:
+// at rotation R, plane k-2+d lives in w[(R+d)%5] (d = 0..4) and its own
+// rho_i / square in ra/sa[(R+d)%5].  R is a template constant in step<R>, so
+// the rotation is pure register renaming (no moves).
+struct Seg {
+    const double *su;
+    uint64_t *full;
+    unsigned int *released;
+    const CUtensorMap *umap, *fmap;
+    int i0, j0, ka, kb, uc, ocol, tx, ty;
+    bool in_grid, active, mid_x, mid_y;
+    Cases cx, cy;
+    uint32_t seq0;
+    double w[5][5];
+    double ra[5], sa[5];
+};
+
+template <int R>
+__device__ __forceinline__ void rhs_step(Seg &g, const Params &P, int k) {
+    constexpr int QQ = R % 5, Q = (R + 1) % 5, Z = (R + 2) % 5, PI = (R + 3) % 5, PP = (R + 4) % 5;
+    const unsigned FULL = 0xffffffffu;
+    const Coef &C = P.c;
+    const uint32_t sq_k = g.seq0 + (uint32_t)(k - g.ka);
+    const double *s = g.su + (size_t)(sq_k % STAGES) * SLOT;
+
+    // forcing(k): staged by the same TMA as plane k (reuse count 1, so it only
+    // needs latency hiding, not a register slot)
+    double acc[5];
+    {
+        const double *fs = s + U_SLOT;
+#pragma unroll
+        for (int m = 0; m < 5; ++m) acc[m] = fs[(m * TY + g.ty) * FX + g.tx + 1];
+    }
+    // own column u(k+2) into the window; own rho_i / square of plane k+1
+    wait_plane(g.full, sq_k + 2);
+    load5(g.w[PP], g.su + (size_t)((sq_k + 2) % STAGES) * SLOT, g.uc);
+    if (g.in_grid) aux_of(g.w[PI][0], g.w[PI][1], g.w[PI][2], g.w[PI][3], g.ra[PI], g.sa[PI]);
+    else { g.ra[PI] = 0.0; g.sa[PI] = 0.0; }
+
+    const double (&wz)[5] = g.w[Z];
+    const double r0 = g.ra[Z], s0 = g.sa[Z];
+    double vc[3];
+    vc[0] = wz[1] * r0;
+    vc[1] = wz[2] * r0;
+    vc[2] = wz[3] * r0;
+    const double qsc = s0 * r0;
+    const double pc = wz[4] * r0;
+    double six[5];
+#pragma unroll
+    for (int m = 0; m < 5; ++m) six[m] = 6.0 * wz[m];
+
+    // xi: rho_i/square of i+-1 are the neighbour lanes' own values; lanes 0
+    // and 31 evaluate their outside neighbour themselves.
+    {
+        Nb p, q;
+        load5(p.u, s, g.uc + 1);
+        load5(q.u, s, g.uc - 1);
+        p.rho = __shfl_down_sync(FULL, r0, 1);
+        p.sq = __shfl_down_sync(FULL, s0, 1);
+        q.rho = __shfl_up_sync(FULL, r0, 1);
+        q.sq = __shfl_up_sync(FULL, s0, 1);
+        {
+            const bool left = (g.tx == 0);
+            double re, se;
+            aux_of(left ? q.u[0] : p.u[0], left ? q.u[1] : p.u[1], left ? q.u[2] : p.u[2],
+                   left ? q.u[3] : p.u[3], re, se);
+            if (left) { q.rho = re; q.sq = se; }
+            if (g.tx == TX - 1) { p.rho = re; p.sq = se; }
+        }
+        flux_dir<1>(acc, wz, vc, qsc, pc, p, q, C, 0);
+        double pp[5], qq[5];
+        load5(pp, s, g.uc + 2);
+        load5(qq, s, g.uc - 2);
+        if (g.mid_x) diss_dir<false>(acc, qq, q.u, wz, six, p.u, pp, C.dssp, g.cx);
+        else diss_dir<true>(acc, qq, q.u, wz, six, p.u, pp, C.dssp, g.cx);
+    }
+    // eta: rows j+-1 belong to other warps; evaluate their rho_i / square
+    // from the u values loaded for the stencil.
+    {
+        Nb p, q;
+        load5(p.u, s, g.uc + UX);
+        load5(q.u, s, g.uc - UX);
+        aux_of(p.u[0], p.u[1], p.u[2], p.u[3], p.rho, p.sq);
+        aux_of(q.u[0], q.u[1], q.u[2], q.u[3], q.rho, q.sq);
+        flux_dir<2>(acc, wz, vc, qsc, pc, p, q, C, 1);
+        double pp[5], qq[5];
+        load5(pp, s, g.uc + 2 * UX);
+        load5(qq, s, g.uc - 2 * UX);
+        if (g.mid_y) diss_dir<false>(acc, qq, q.u, wz, six, p.u, pp, C.dssp, g.cy);
+        else diss_dir<true>(acc, qq, q.u, wz, six, p.u, pp, C.dssp, g.cy);
+    }
+    // zeta: everything from the register window (inter-iteration scalar
+    // replacement along the sequential loop)
+    {
+        Nb p, q;
+#pragma unroll
+        for (int m = 0; m < 5; ++m) {
+            p.u[m] = g.w[PI][m];
+            q.u[m] = g.w[Q][m];
+        }
+        p.rho = g.ra[PI]; p.sq = g.sa[PI];
+        q.rho = g.ra[Q]; q.sq = g.sa[Q];
+        flux_dir<3>(acc, wz, vc, qsc, pc, p, q, C, 2);
+        if (is_mid(k, P.nz))
+            diss_dir<false>(acc, g.w[QQ], g.w[Q], wz, six, g.w[PI], g.w[PP], C.dssp, Cases{});
+        else
+            diss_dir<true>(acc, g.w[QQ], g.w[Q], wz, six, g.w[PI], g.w[PP], C.dssp,
+                           cases_of(k, P.nz));
+    }
+    if (g.active) {
+        const int o = g.ocol + P.sk * (k - P.k0);
+#pragma unroll
+        for (int m = 0; m < 5; ++m) __stcs(P.r + o + P.sm * m, acc[m] * C.dt);
+    }
+    // release plane k's slot; the last warp out refills it with plane k+STAGES
+    __syncwarp();
+    if (g.tx == 0) {
+        const int slot = (int)(sq_k % STAGES);
+        __threadfence_block();
+        const unsigned old = atomicAdd(&g.released[slot], 1u);
+        if (old == (unsigned)(TY - 1)) {
+            g.released[slot] = 0;
+            __threadfence_block();
+            const int kn = k + STAGES;
+            if (kn <= g.kb + 1)
+                issue_plane(g.umap, g.fmap, P, const_cast<double *>(g.su), g.full, g.i0, g.j0, kn,
+                            kn < g.kb, sq_k + STAGES);
+        }
+    }
 }
 
 // One CTA processes the column-plane units [blockIdx*units/ncta, ...).
 // Warps are decoupled: warp w owns row j0+w of the tile and never waits for
 // another warp except through the TMA ring (a slot is refilled by the last
 // warp to release it).
-__device__ __forceinline__ void rhs_body(const CUtensorMap *tmap, const Params &P) {
+__device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensorMap *fmap,
+                                         const Params &P) {
     extern __shared__ __align__(128) unsigned char smem_raw[];
     double *su = reinterpret_cast<double *>(smem_raw);
-    uint64_t *full = reinterpret_cast<uint64_t *>(su + (size_t)STAGES * U_SLOT);
+    uint64_t *full = reinterpret_cast<uint64_t *>(su + (size_t)STAGES * SLOT);
     unsigned int *released = reinterpret_cast<unsigned int *>(full + STAGES);
 
     const int tid = threadIdx.x;
-    const int tx = tid % TX, ty = tid / TX;  // lane = tx, warp = ty
-    const unsigned FULL = 0xffffffffu;
-    const Coef &C = P.c;
 
     if (tid == 0) {
-        prefetch_tmap(tmap);
+        prefetch_tmap(umap);
+        prefetch_tmap(fmap);
         for (int s = 0; s < STAGES; ++s) {
             mbar_init(&full[s], 1);
             released[s] = 0;
@@ -311,210 +458,88 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *tmap, const Params &
 
     copy_faces(P);
 
-    long long ub = (long long)blockIdx.x * P.units / P.ncta;
-    const long long ue = (long long)(blockIdx.x + 1) * P.units / P.ncta;
-    uint32_t seq0 = 0;
+    int ub = split_point((int)blockIdx.x, P.units, P.ncta);
+    const int ue = split_point((int)blockIdx.x + 1, P.units, P.ncta);
+
+    Seg g;
+    g.su = su;
+    g.full = full;
+    g.released = released;
+    g.umap = umap;
+    g.fmap = fmap;
+    g.tx = tid % TX;
+    g.ty = tid / TX;  // lane = tx, warp = ty
+    g.seq0 = 0;
 
     while (ub < ue) {
         // ---- segment: one column tile, a contiguous run of planes ----
         int col, pidx, run;
         decode_unit(P, ub, col, pidx, run);
-        int ka, kb;
         {
-            const long long left = min((long long)run, ue - ub);
+            const int left = min(run, ue - ub);
             if (pidx < P.n0) {
-                ka = P.ka0 + pidx;
-                kb = (int)min((long long)P.kb0, ka + left);
+                g.ka = P.ka0 + pidx;
+                g.kb = min(P.kb0, g.ka + left);
             } else {
-                ka = P.ka1 + (pidx - P.n0);
-                kb = (int)min((long long)P.kb1, ka + left);
+                g.ka = P.ka1 + (pidx - P.n0);
+                g.kb = min(P.kb1, g.ka + left);
             }
         }
-        ub += kb - ka;
+        ub += g.kb - g.ka;
+        const int ka = g.ka, kb = g.kb;
 
-        const int i0 = 1 + (col % P.ntx) * TX;
-        const int j0 = 1 + (col / P.ntx) * TY;
-        const int i = i0 + tx, j = j0 + ty;
-        const bool in_grid = (i < P.nx) && (j < P.ny);
-        const bool active = (i <= P.nx - 2) && (j <= P.ny - 2);
+        g.i0 = 1 + (col % P.ntx) * TX;
+        g.j0 = 1 + (col / P.ntx) * TY;
+        const int i = g.i0 + g.tx, j = g.j0 + g.ty;
+        g.in_grid = (i < P.nx) && (j < P.ny);
+        g.active = (i <= P.nx - 2) && (j <= P.ny - 2);
         const int nload = kb - ka + 2;  // planes ka .. kb+1
 
         if (tid == 0) {
             const int npre = nload < STAGES ? nload : STAGES;
-            for (int s = 0; s < npre; ++s) issue_plane(tmap, P, su, full, i0, j0, ka + s, seq0 + s);
+            for (int s = 0; s < npre; ++s)
+                issue_plane(umap, fmap, P, su, full, g.i0, g.j0, ka + s, ka + s < kb, g.seq0 + s);
         }
 
         // Case flags (global indices, reading c12).
-        const bool mid_x = is_mid(i0, P.nx) && is_mid(i0 + TX - 1, P.nx);
-        const bool mid_y = is_mid(j, P.ny);
-        const Cases cx = cases_of(i, P.nx), cy = cases_of(j, P.ny);
+        g.mid_x = is_mid(g.i0, P.nx) && is_mid(g.i0 + TX - 1, P.nx);
+        g.mid_y = is_mid(j, P.ny);
+        g.cx = cases_of(i, P.nx);
+        g.cy = cases_of(j, P.ny);
+        g.uc = (g.ty + 2) * UX + (g.tx + HX);  // centre in the u tile
+        g.ocol = i + P.sy * j;                  // own column offset (dim)
 
-        const int uc = (ty + 2) * UX + (tx + HX);  // centre in the u tile
-        const int ocol = i + P.sy * j;             // own column offset (dim)
-
-        // Register window u(:, k-2..k+2) and own rho_i/square at k-1..k+1.
-        double w0[5], w1[5], w2[5], w3[5], w4[5];
-        double rm1, sm1, r0, s0, rp1, sp1;
+        // Window at rotation 0: planes ka-2, ka-1 from global memory (read
+        // once per segment), ka and ka+1 from the TMA ring.
         {
             const int kbm2 = ka - 2 - P.k0 + P.ukoff, kbm1 = ka - 1 - P.k0 + P.ukoff;
 #pragma unroll
             for (int m = 0; m < 5; ++m) {
-                w0[m] = (in_grid && kbm2 >= 0) ? __ldg(P.u + ocol + P.sm * m + P.sk * kbm2) : 0.0;
-                w1[m] = (in_grid && kbm1 >= 0) ? __ldg(P.u + ocol + P.sm * m + P.sk * kbm1) : 0.0;
+                g.w[0][m] = (g.in_grid && kbm2 >= 0) ? __ldg(P.u + g.ocol + P.sm * m + P.sk * kbm2) : 0.0;
+                g.w[1][m] = (g.in_grid && kbm1 >= 0) ? __ldg(P.u + g.ocol + P.sm * m + P.sk * kbm1) : 0.0;
             }
-            if (in_grid && kbm1 >= 0) aux_of(w1[0], w1[1], w1[2], w1[3], rm1, sm1);
-            else { rm1 = 0.0; sm1 = 0.0; }
+            if (g.in_grid && kbm1 >= 0) aux_of(g.w[1][0], g.w[1][1], g.w[1][2], g.w[1][3], g.ra[1], g.sa[1]);
+            else { g.ra[1] = 0.0; g.sa[1] = 0.0; }
         }
-        wait_plane(full, seq0);
-        load5(w2, su + (size_t)(seq0 % STAGES) * U_SLOT, uc);
-        if (in_grid) aux_of(w2[0], w2[1], w2[2], w2[3], r0, s0);
-        else { r0 = 0.0; s0 = 0.0; }
-        wait_plane(full, seq0 + 1);
-        load5(w3, su + (size_t)((seq0 + 1) % STAGES) * U_SLOT, uc);
+        wait_plane(full, g.seq0);
+        load5(g.w[2], su + (size_t)(g.seq0 % STAGES) * SLOT, g.uc);
+        if (g.in_grid) aux_of(g.w[2][0], g.w[2][1], g.w[2][2], g.w[2][3], g.ra[2], g.sa[2]);
+        else { g.ra[2] = 0.0; g.sa[2] = 0.0; }
+        wait_plane(full, g.seq0 + 1);
+        load5(g.w[3], su + (size_t)((g.seq0 + 1) % STAGES) * SLOT, g.uc);
 
-#if SAFARA_FPREFETCH
-        double fn[5];
-        {
-            const int kl = ka - P.k0;
-#pragma unroll
-            for (int m = 0; m < 5; ++m)
-                fn[m] = active ? __ldcs(P.f + ocol + P.sm * m + P.sk * kl) : 0.0;
+        for (int k = ka; k < kb; k += 5) {
+            rhs_step<0>(g, P, k);
+            if (k + 1 >= kb) break;
+            rhs_step<1>(g, P, k + 1);
+            if (k + 2 >= kb) break;
+            rhs_step<2>(g, P, k + 2);
+            if (k + 3 >= kb) break;
+            rhs_step<3>(g, P, k + 3);
+            if (k + 4 >= kb) break;
+            rhs_step<4>(g, P, k + 4);
         }
-#endif
-
-        for (int k = ka; k < kb; ++k) {
-            const uint32_t sq_k = seq0 + (uint32_t)(k - ka);
-            // forcing is used once (reuse count 1): streamed, never staged.
-            double fr[5];
-#if SAFARA_FPREFETCH
-            // prefetched one step ahead; stream forcing(k+1)
-#pragma unroll
-            for (int m = 0; m < 5; ++m) fr[m] = fn[m];
-            {
-                const int kl = k + 1 - P.k0;
-                const bool ok = active && (k + 1 < kb);
-#pragma unroll
-                for (int m = 0; m < 5; ++m)
-                    fn[m] = ok ? __ldcs(P.f + ocol + P.sm * m + P.sk * kl) : 0.0;
-            }
-#else
-            {
-                const int kl = k - P.k0;
-#pragma unroll
-                for (int m = 0; m < 5; ++m)
-                    fr[m] = active ? __ldcs(P.f + ocol + P.sm * m + P.sk * kl) : 0.0;
-            }
-#endif
-            // own column u(k+2) into the window; own rho_i/square of plane k+1
-            wait_plane(full, sq_k + 2);
-            load5(w4, su + (size_t)((sq_k + 2) % STAGES) * U_SLOT, uc);
-            if (in_grid) aux_of(w3[0], w3[1], w3[2], w3[3], rp1, sp1);
-            else { rp1 = 0.0; sp1 = 0.0; }
-
-            // ---- the point (i, j, k): every lane runs it (shuffles), only
-            // active lanes store ----
-            {
-                const double *s = su + (size_t)(sq_k % STAGES) * U_SLOT;
-
-                double acc[5];
-#pragma unroll
-                for (int m = 0; m < 5; ++m) acc[m] = fr[m];
-
-                double vc[3];
-                vc[0] = w2[1] * r0;
-                vc[1] = w2[2] * r0;
-                vc[2] = w2[3] * r0;
-                const double qsc = s0 * r0;
-                const double pc = w2[4] * r0;
-                double six[5];
-#pragma unroll
-                for (int m = 0; m < 5; ++m) six[m] = 6.0 * w2[m];
-
-                // xi: rho_i/square of i+-1 are the neighbour lanes' own values;
-                // lanes 0 and 31 evaluate their outside neighbour themselves.
-                {
-                    Nb p, q;
-                    load5(p.u, s, uc + 1);
-                    load5(q.u, s, uc - 1);
-                    p.rho = __shfl_down_sync(FULL, r0, 1);
-                    p.sq = __shfl_down_sync(FULL, s0, 1);
-                    q.rho = __shfl_up_sync(FULL, r0, 1);
-                    q.sq = __shfl_up_sync(FULL, s0, 1);
-                    {
-                        const bool left = (tx == 0);
-                        double re, se;
-                        aux_of(left ? q.u[0] : p.u[0], left ? q.u[1] : p.u[1],
-                               left ? q.u[2] : p.u[2], left ? q.u[3] : p.u[3], re, se);
-                        if (left) { q.rho = re; q.sq = se; }
-                        if (tx == TX - 1) { p.rho = re; p.sq = se; }
-                    }
-                    flux_dir<1>(acc, w2, vc, qsc, pc, p, q, C, 0);
-                    double pp[5], qq[5];
-                    load5(pp, s, uc + 2);
-                    load5(qq, s, uc - 2);
-                    if (mid_x) diss_dir<false>(acc, qq, q.u, w2, six, p.u, pp, C.dssp, cx);
-                    else diss_dir<true>(acc, qq, q.u, w2, six, p.u, pp, C.dssp, cx);
-                }
-                // eta: rows j+-1 belong to other warps; evaluate their
-                // rho_i/square from the u values loaded for the stencil.
-                {
-                    Nb p, q;
-                    load5(p.u, s, uc + UX);
-                    load5(q.u, s, uc - UX);
-                    aux_of(p.u[0], p.u[1], p.u[2], p.u[3], p.rho, p.sq);
-                    aux_of(q.u[0], q.u[1], q.u[2], q.u[3], q.rho, q.sq);
-                    flux_dir<2>(acc, w2, vc, qsc, pc, p, q, C, 1);
-                    double pp[5], qq[5];
-                    load5(pp, s, uc + 2 * UX);
-                    load5(qq, s, uc - 2 * UX);
-                    if (mid_y) diss_dir<false>(acc, qq, q.u, w2, six, p.u, pp, C.dssp, cy);
-                    else diss_dir<true>(acc, qq, q.u, w2, six, p.u, pp, C.dssp, cy);
-                }
-                // zeta: everything from the register window
-                {
-                    Nb p, q;
-#pragma unroll
-                    for (int m = 0; m < 5; ++m) {
-                        p.u[m] = w3[m];
-                        q.u[m] = w1[m];
-                    }
-                    p.rho = rp1; p.sq = sp1;
-                    q.rho = rm1; q.sq = sm1;
-                    flux_dir<3>(acc, w2, vc, qsc, pc, p, q, C, 2);
-                    if (is_mid(k, P.nz)) diss_dir<false>(acc, w0, w1, w2, six, w3, w4, C.dssp, Cases{});
-                    else diss_dir<true>(acc, w0, w1, w2, six, w3, w4, C.dssp, cases_of(k, P.nz));
-                }
-                if (active) {
-                    const int o = ocol + P.sk * (k - P.k0);
-#pragma unroll
-                    for (int m = 0; m < 5; ++m) __stcs(P.r + o + P.sm * m, acc[m] * C.dt);
-                }
-            }
-            // release plane k's slot; the last warp out refills it with k+STAGES
-            __syncwarp();
-            if (tx == 0) {
-                const int slot = (int)(sq_k % STAGES);
-                __threadfence_block();
-                const unsigned old = atomicAdd(&released[slot], 1u);
-                if (old == (unsigned)(TY - 1)) {
-                    released[slot] = 0;
-                    __threadfence_block();
-                    const int kn = k + STAGES;
-                    if (kn <= kb + 1) issue_plane(tmap, P, su, full, i0, j0, kn, sq_k + STAGES);
-                }
-            }
-            // rotate the windows
-#pragma unroll
-            for (int m = 0; m < 5; ++m) {
-                w0[m] = w1[m];
-                w1[m] = w2[m];
-                w2[m] = w3[m];
-                w3[m] = w4[m];
-            }
-            rm1 = r0; sm1 = s0;
-            r0 = rp1; s0 = sp1;
-        }
-        seq0 += (uint32_t)nload;
+        g.seq0 += (uint32_t)nload;
         // Segment end: every warp has consumed every plane; planes kb, kb+1
         // were never released, so clear the counters before the next segment.
         __syncthreads();

@@ -26,7 +26,13 @@ constexpr int UY = TY + 4;           // u tile incl. j halo of 2
 constexpr int U_PLANE = UX * UY * 5; // doubles in one TMA box (one u plane tile)
 constexpr int U_SLOT = ((U_PLANE * 8 + 127) / 128) * 128 / 8;  // slot stride: TMA dst 128 B aligned
 constexpr uint32_t TMA_BYTES = U_PLANE * 8u;
-constexpr size_t SMEM_BYTES = (size_t)STAGES * U_SLOT * 8 + STAGES * 8 + STAGES * 4;
+// forcing tile of the same plane: i0-1 .. i0+TX (16-byte aligned start), no j halo
+constexpr int FX = TX + 2;
+constexpr int F_PLANE = FX * TY * 5;
+constexpr int F_SLOT = ((F_PLANE * 8 + 127) / 128) * 128 / 8;
+constexpr uint32_t TMA_BYTES_F = F_PLANE * 8u;
+constexpr int SLOT = U_SLOT + F_SLOT;  // doubles per ring slot: u tile then forcing tile
+constexpr size_t SMEM_BYTES = (size_t)STAGES * SLOT * 8 + STAGES * 8 + STAGES * 4;
 constexpr int MIN_PLANES_PER_CTA = 4;
 
 // Device-side coefficients: safara_coeffs_t plus the constant products that
@@ -50,7 +56,7 @@ struct Params {
     int ncol;              // ntx * nty
     int chunk;             // planes per chunk of the chunk-major unit order
     int ncta;              // CTAs in the grid
-    long long units;       // ntx*nty*nplanes (column-plane work items)
+    int units;             // ncol*nplanes (column-plane work items, < 2^31)
     int fk_lo, fk_hi;      // local planes whose boundary faces this launch copies
     int pos_j, pos_m, pos_k;  // tensor-map dimension holding j, m, k
     const double *u;       // u buffer base (local plane 0)
@@ -60,8 +66,10 @@ struct Params {
 };
 
 // Launchers implemented in rhs_fast.cu / rhs_strict.cu.
-cudaError_t launch_rhs_fast(const CUtensorMap &tmap, const Params &p, cudaStream_t s);
-cudaError_t launch_rhs_strict(const CUtensorMap &tmap, const Params &p, cudaStream_t s);
+cudaError_t launch_rhs_fast(const CUtensorMap &umap, const CUtensorMap &fmap, const Params &p,
+                            cudaStream_t s);
+cudaError_t launch_rhs_strict(const CUtensorMap &umap, const CUtensorMap &fmap, const Params &p,
+                              cudaStream_t s);
 cudaError_t setup_rhs_fast(int *ctas_per_sm, cudaFuncAttributes *attr);
 cudaError_t setup_rhs_strict(int *ctas_per_sm, cudaFuncAttributes *attr);
 
