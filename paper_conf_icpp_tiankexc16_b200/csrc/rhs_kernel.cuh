@@ -33,6 +33,10 @@
 
 #include "safara_internal.h"
 
+#ifndef SAFARA_SIX_ARRAY
+#define SAFARA_SIX_ARRAY 0
+#endif
+
 
 namespace safara {
 namespace dev {
@@ -176,6 +180,11 @@ __device__ __forceinline__ Cases cases_of(int x, int n) {
 
 __device__ __forceinline__ bool is_mid(int x, int n) { return x >= 3 && x <= n - 4; }
 
+#if SAFARA_SIX_ARRAY
+#define SIXOF(m) six[m]
+#else
+#define SIXOF(m) (6.0 * a0[m])
+#endif
 template <bool GENERIC>
 __device__ __forceinline__ void diss_dir(double (&acc)[5], const double (&am2)[5],
                                          const double (&am1)[5], const double (&a0)[5],
@@ -186,7 +195,7 @@ __device__ __forceinline__ void diss_dir(double (&acc)[5], const double (&am2)[5
         double t;
         if (!GENERIC) {
             t = __fma_rn(-4.0, am1[m], am2[m]);
-            t = t + six[m];
+            t = t + SIXOF(m);
             t = __fma_rn(-4.0, ap1[m], t);
             t = t + ap2[m];
         } else {
@@ -194,7 +203,7 @@ __device__ __forceinline__ void diss_dir(double (&acc)[5], const double (&am2)[5
             const double x1 = cs.hm1 ? am1[m] : 0.0;
             const double y1 = cs.hp1 ? ap1[m] : 0.0;
             const double y2 = cs.hp2 ? ap2[m] : 0.0;
-            const double cc = cs.five ? 5.0 * a0[m] : six[m];
+            const double cc = cs.five ? 5.0 * a0[m] : SIXOF(m);
             t = __fma_rn(-4.0, x1, x2);
             t = t + cc;
             t = __fma_rn(-4.0, y1, t);
@@ -303,8 +312,9 @@ __device__ __forceinline__ void decode_unit(const Params &P, int L, int &col, in
 
 // Per-segment state of one thread.  The register window is a 5-entry ring:
 // at rotation R, plane k-2+d lives in w[(R+d)%5] (d = 0..4) and its own
-// rho_i / square in ra/sa[(R+d)%5].  R is a template constant in step<R>, so
-// the rotation is pure register renaming (no moves).
+// rho_i / square in ra/sa[(R+d)%5].  step<R> supports pure register renaming
+// (unroll by 5); the loop uses R = 0 plus explicit moves, which measured
+// faster because the 5x unrolled body overflows the instruction cache.
 struct Seg {
     const double *su;
     uint64_t *full;
@@ -348,9 +358,13 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, int k) {
     vc[2] = wz[3] * r0;
     const double qsc = s0 * r0;
     const double pc = wz[4] * r0;
+#if SAFARA_SIX_ARRAY
     double six[5];
 #pragma unroll
     for (int m = 0; m < 5; ++m) six[m] = 6.0 * wz[m];
+#else
+    const double(&six)[5] = wz;  // unused: diss_dir forms 6.0*a0 itself
+#endif
 
     // xi: rho_i/square of i+-1 are the neighbour lanes' own values; lanes 0
     // and 31 evaluate their outside neighbour themselves.
@@ -528,16 +542,17 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensor
         wait_plane(full, g.seq0 + 1);
         load5(g.w[3], su + (size_t)((g.seq0 + 1) % STAGES) * SLOT, g.uc);
 
-        for (int k = ka; k < kb; k += 5) {
+        // One step body (instruction-cache footprint) and a register-move
+        // rotation; unrolling by 5 for pure renaming measured slower (I$).
+        for (int k = ka; k < kb; ++k) {
             rhs_step<0>(g, P, k);
-            if (k + 1 >= kb) break;
-            rhs_step<1>(g, P, k + 1);
-            if (k + 2 >= kb) break;
-            rhs_step<2>(g, P, k + 2);
-            if (k + 3 >= kb) break;
-            rhs_step<3>(g, P, k + 3);
-            if (k + 4 >= kb) break;
-            rhs_step<4>(g, P, k + 4);
+#pragma unroll
+            for (int d = 0; d < 4; ++d) {
+#pragma unroll
+                for (int m = 0; m < 5; ++m) g.w[d][m] = g.w[d + 1][m];
+                g.ra[d] = g.ra[d + 1];
+                g.sa[d] = g.sa[d + 1];
+            }
         }
         g.seq0 += (uint32_t)nload;
         // Segment end: every warp has consumed every plane; planes kb, kb+1
