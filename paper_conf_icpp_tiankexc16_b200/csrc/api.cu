@@ -185,13 +185,17 @@ int launch(const double *u, const double *f, double *r, const safara_dims_t &d, 
     const int per_sm = strict ? st.ctas_strict : st.ctas_fast;
     const long long max_ctas = (long long)std::max(per_sm, 1) * st.sms;
     long long ncta;
-    if (g_tune.sched == 1 && p.ncol <= max_ctas && p.nplanes > 0) {
-        // Lockstep: every CTA owns one (column tile, k-part) and all parts
-        // start together, so neighbouring tiles read a plane's shared halo
-        // at the same time and the second read hits L2.
-        long long parts = max_ctas / p.ncol;
-        parts = std::min<long long>(parts, std::max(1, p.nplanes / MIN_PLANES_PER_CTA));
-        ncta = p.ncol * std::max<long long>(parts, 1);
+    long long parts = p.ncol > 0 ? max_ctas / p.ncol : 0;
+    parts = std::min<long long>(parts, std::max(1, p.nplanes / MIN_PLANES_PER_CTA));
+    // Lockstep only when it keeps >= 90% of the CTA slots busy (e.g. class C:
+    // 70 column tiles x 2 parts = 140 of 148); otherwise balanced ranges.
+    const bool lockstep = g_tune.sched == 1 && parts >= 1 && p.nplanes > 0 &&
+                          (parts * p.ncol * 10 >= 9 * std::min<long long>(max_ctas, p.units));
+    if (lockstep) {
+        // Every CTA owns one (column tile, k-part) and all parts start
+        // together, so neighbouring tiles read a plane's shared halo at the
+        // same time and the second read hits L2.
+        ncta = p.ncol * parts;
     } else {
         ncta = (p.units + MIN_PLANES_PER_CTA - 1) / MIN_PLANES_PER_CTA;
         ncta = std::min(ncta, max_ctas);

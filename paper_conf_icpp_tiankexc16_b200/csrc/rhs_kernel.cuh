@@ -33,8 +33,8 @@
 
 #include "safara_internal.h"
 
-#ifndef SAFARA_SIX_ARRAY
-#define SAFARA_SIX_ARRAY 0
+#ifndef SAFARA_L2PF
+#define SAFARA_L2PF 0  // planes beyond the ring to prefetch into L2 (0 = off)
 #endif
 
 
@@ -76,6 +76,10 @@ __device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
     } while (!done);
 }
 
+__device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+
 __device__ __forceinline__ void tma_load_4d(void *dst, const CUtensorMap *map, uint64_t *bar,
                                             int c0, int c1, int c2, int c3) {
     asm volatile(
@@ -83,6 +87,15 @@ __device__ __forceinline__ void tma_load_4d(void *dst, const CUtensorMap *map, u
         " [%0], [%1, {%2, %3, %4, %5}], [%6];" ::"r"(smem_u32(dst)),
         "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(c2), "r"(c3),
         "r"(smem_u32(bar))
+        : "memory");
+}
+
+__device__ __forceinline__ void tma_prefetch_l2_4d(const CUtensorMap *map, int c0, int c1, int c2,
+                                                   int c3) {
+    asm volatile(
+        "cp.async.bulk.prefetch.tensor.4d.L2.global.tile [%0, {%1, %2, %3, %4}];" ::"l"(
+            reinterpret_cast<uint64_t>(map)),
+        "r"(c0), "r"(c1), "r"(c2), "r"(c3)
         : "memory");
 }
 
@@ -96,10 +109,29 @@ __device__ __forceinline__ double d2(double ap, double ac, double aq) {
     return __fma_rn(-2.0, ac, ap) + aq;
 }
 
+// Reciprocal.  STRICT: IEEE 1.0/x (correctly rounded, bit-identical to the
+// oracle).  Production: MUFU.RCP64H seed + three Newton steps, branch-free
+// (<= 1 ulp for the normal, positive densities of the path; the IEEE
+// division's special-case branch costs ~6 issue slots per call).
+__device__ __forceinline__ double recip(double x) {
+#if SAFARA_STRICT_BUILD
+    return 1.0 / x;
+#else
+    double r;
+    asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(r) : "d"(x));
+    double e = __fma_rn(-x, r, 1.0);
+    r = __fma_rn(r, e, r);
+    e = __fma_rn(-x, r, 1.0);
+    r = __fma_rn(r, e, r);
+    e = __fma_rn(-x, r, 1.0);
+    return __fma_rn(r, e, r);
+#endif
+}
+
 // rho_i = 1.0/u1; square = 0.5*(u2*u2 + u3*u3 + u4*u4)*rho_i  (App. A step 0)
 __device__ __forceinline__ void aux_of(double u1, double u2, double u3, double u4, double &rho,
                                        double &sq) {
-    rho = 1.0 / u1;
+    rho = recip(u1);
     sq = 0.5 * (u2 * u2 + u3 * u3 + u4 * u4) * rho;
 }
 
@@ -180,37 +212,38 @@ __device__ __forceinline__ Cases cases_of(int x, int n) {
 
 __device__ __forceinline__ bool is_mid(int x, int n) { return x >= 3 && x <= n - 4; }
 
-#if SAFARA_SIX_ARRAY
-#define SIXOF(m) six[m]
-#else
-#define SIXOF(m) (6.0 * a0[m])
-#endif
+// The dissipation stencil value t_m (before `rhs -= dssp*t`).  It is formed
+// ahead of the flux terms (so the i+-2 / j+-2 neighbours die early: register
+// pressure) and subtracted after them, keeping the NAS accumulation order.
 template <bool GENERIC>
-__device__ __forceinline__ void diss_dir(double (&acc)[5], const double (&am2)[5],
-                                         const double (&am1)[5], const double (&a0)[5],
-                                         const double (&six)[5], const double (&ap1)[5],
-                                         const double (&ap2)[5], double dssp, Cases cs) {
+__device__ __forceinline__ void diss_terms(double (&t)[5], const double (&am2)[5],
+                                           const double (&am1)[5], const double (&a0)[5],
+                                           const double (&ap1)[5], const double (&ap2)[5],
+                                           Cases cs) {
 #pragma unroll
     for (int m = 0; m < 5; ++m) {
-        double t;
         if (!GENERIC) {
-            t = __fma_rn(-4.0, am1[m], am2[m]);
-            t = t + SIXOF(m);
-            t = __fma_rn(-4.0, ap1[m], t);
-            t = t + ap2[m];
+            t[m] = __fma_rn(-4.0, am1[m], am2[m]);
+            t[m] = t[m] + 6.0 * a0[m];
+            t[m] = __fma_rn(-4.0, ap1[m], t[m]);
+            t[m] = t[m] + ap2[m];
         } else {
             const double x2 = cs.hm2 ? am2[m] : 0.0;
             const double x1 = cs.hm1 ? am1[m] : 0.0;
             const double y1 = cs.hp1 ? ap1[m] : 0.0;
             const double y2 = cs.hp2 ? ap2[m] : 0.0;
-            const double cc = cs.five ? 5.0 * a0[m] : SIXOF(m);
-            t = __fma_rn(-4.0, x1, x2);
-            t = t + cc;
-            t = __fma_rn(-4.0, y1, t);
-            t = t + y2;
+            const double cc = cs.five ? 5.0 * a0[m] : 6.0 * a0[m];
+            t[m] = __fma_rn(-4.0, x1, x2);
+            t[m] = t[m] + cc;
+            t[m] = __fma_rn(-4.0, y1, t[m]);
+            t[m] = t[m] + y2;
         }
-        acc[m] = acc[m] - dssp * t;
     }
+}
+
+__device__ __forceinline__ void diss_apply(double (&acc)[5], const double (&t)[5], double dssp) {
+#pragma unroll
+    for (int m = 0; m < 5; ++m) acc[m] = acc[m] - dssp * t[m];
 }
 
 // Copy forcing -> rhs on this launch's boundary-face points (rhs = forcing,
@@ -252,8 +285,11 @@ __device__ __forceinline__ void copy_faces(const Params &P) {
             j = 1 + r / (nx - 2);
         }
         const int o = i + P.sy * j + P.sk * kl;
+        double v[5];  // all loads first: rhs may not alias forcing (ABI), but
+#pragma unroll    // the compiler cannot know that
+        for (int m = 0; m < 5; ++m) v[m] = __ldcs(P.f + o + P.sm * m);
 #pragma unroll
-        for (int m = 0; m < 5; ++m) __stcs(P.r + o + P.sm * m, __ldcs(P.f + o + P.sm * m));
+        for (int m = 0; m < 5; ++m) __stcs(P.r + o + P.sm * m, v[m]);
     }
 }
 
@@ -278,6 +314,22 @@ __device__ __forceinline__ void issue_plane(const CUtensorMap *umap, const CUten
         const int f3 = P.pos_j == 3 ? j0 : (P.pos_m == 3 ? 0 : kf);
         tma_load_4d(dst + U_SLOT, fmap, &full[slot], i0 - 1, f1, f2, f3);
     }
+}
+
+// Warm L2 with plane k's u and forcing boxes (no smem, no barrier).
+__device__ __forceinline__ void prefetch_plane_l2(const CUtensorMap *umap, const CUtensorMap *fmap,
+                                                  const Params &P, int i0, int j0, int k,
+                                                  bool with_f) {
+    const int kb = k - P.k0 + P.ukoff;
+    const int kf = k - P.k0;
+    const int jc = j0 - 2;
+    tma_prefetch_l2_4d(umap, i0 - HX, P.pos_j == 1 ? jc : (P.pos_m == 1 ? 0 : kb),
+                       P.pos_j == 2 ? jc : (P.pos_m == 2 ? 0 : kb),
+                       P.pos_j == 3 ? jc : (P.pos_m == 3 ? 0 : kb));
+    if (with_f)
+        tma_prefetch_l2_4d(fmap, i0 - 1, P.pos_j == 1 ? j0 : (P.pos_m == 1 ? 0 : kf),
+                           P.pos_j == 2 ? j0 : (P.pos_m == 2 ? 0 : kf),
+                           P.pos_j == 3 ? j0 : (P.pos_m == 3 ? 0 : kf));
 }
 
 __device__ __forceinline__ void wait_plane(uint64_t *full, uint32_t seq) {
@@ -310,31 +362,55 @@ __device__ __forceinline__ void decode_unit(const Params &P, int L, int &col, in
     run = kc - off;
 }
 
+// The segment starting at unit ub (not crossing a column, a plane range or
+// the CTA's end ue): column tile `col`, global planes [ka, kb).
+__device__ __forceinline__ void segment_of(const Params &P, int ub, int ue, int &col, int &ka,
+                                           int &kb) {
+    int pidx, run;
+    decode_unit(P, ub, col, pidx, run);
+    const int left = min(run, ue - ub);
+    if (pidx < P.n0) {
+        ka = P.ka0 + pidx;
+        kb = min(P.kb0, ka + left);
+    } else {
+        ka = P.ka1 + (pidx - P.n0);
+        kb = min(P.kb1, ka + left);
+    }
+}
+
 // Per-segment state of one thread.  The register window is a 5-entry ring:
 // at rotation R, plane k-2+d lives in w[(R+d)%5] (d = 0..4) and its own
 // rho_i / square in ra/sa[(R+d)%5].  step<R> supports pure register renaming
 // (unroll by 5); the loop uses R = 0 plus explicit moves, which measured
 // faster because the 5x unrolled body overflows the instruction cache.
+// Shared-memory carve-up (addresses are link-time constants, so nothing here
+// occupies a register across the loop).
+extern __shared__ __align__(128) unsigned char smem_raw[];
+__device__ __forceinline__ double *smem_ring() { return reinterpret_cast<double *>(smem_raw); }
+__device__ __forceinline__ uint64_t *smem_full() {
+    return reinterpret_cast<uint64_t *>(smem_ring() + (size_t)STAGES * SLOT);
+}
+__device__ __forceinline__ unsigned int *smem_released() {
+    return reinterpret_cast<unsigned int *>(smem_full() + STAGES);
+}
+
 struct Seg {
-    const double *su;
-    uint64_t *full;
-    unsigned int *released;
-    const CUtensorMap *umap, *fmap;
     int i0, j0, ka, kb, uc, ocol, tx, ty;
     bool in_grid, active, mid_x, mid_y;
-    Cases cx, cy;
     uint32_t seq0;
     double w[5][5];
     double ra[5], sa[5];
 };
 
 template <int R>
-__device__ __forceinline__ void rhs_step(Seg &g, const Params &P, int k) {
+__device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensorMap *umap,
+                                         const CUtensorMap *fmap, int k) {
     constexpr int QQ = R % 5, Q = (R + 1) % 5, Z = (R + 2) % 5, PI = (R + 3) % 5, PP = (R + 4) % 5;
     const unsigned FULL = 0xffffffffu;
     const Coef &C = P.c;
     const uint32_t sq_k = g.seq0 + (uint32_t)(k - g.ka);
-    const double *s = g.su + (size_t)(sq_k % STAGES) * SLOT;
+    double *const su = smem_ring();
+    const double *s = su + (size_t)(sq_k % STAGES) * SLOT;
 
     // forcing(k): staged by the same TMA as plane k (reuse count 1, so it only
     // needs latency hiding, not a register slot)
@@ -345,11 +421,10 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, int k) {
         for (int m = 0; m < 5; ++m) acc[m] = fs[(m * TY + g.ty) * FX + g.tx + 1];
     }
     // own column u(k+2) into the window; own rho_i / square of plane k+1
-    wait_plane(g.full, sq_k + 2);
-    load5(g.w[PP], g.su + (size_t)((sq_k + 2) % STAGES) * SLOT, g.uc);
+    wait_plane(smem_full(), sq_k + 2);
+    load5(g.w[PP], su + (size_t)((sq_k + 2) % STAGES) * SLOT, g.uc);
     if (g.in_grid) aux_of(g.w[PI][0], g.w[PI][1], g.w[PI][2], g.w[PI][3], g.ra[PI], g.sa[PI]);
     else { g.ra[PI] = 0.0; g.sa[PI] = 0.0; }
-
     const double (&wz)[5] = g.w[Z];
     const double r0 = g.ra[Z], s0 = g.sa[Z];
     double vc[3];
@@ -358,14 +433,6 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, int k) {
     vc[2] = wz[3] * r0;
     const double qsc = s0 * r0;
     const double pc = wz[4] * r0;
-#if SAFARA_SIX_ARRAY
-    double six[5];
-#pragma unroll
-    for (int m = 0; m < 5; ++m) six[m] = 6.0 * wz[m];
-#else
-    const double(&six)[5] = wz;  // unused: diss_dir forms 6.0*a0 itself
-#endif
-
     // xi: rho_i/square of i+-1 are the neighbour lanes' own values; lanes 0
     // and 31 evaluate their outside neighbour themselves.
     {
@@ -384,12 +451,16 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, int k) {
             if (left) { q.rho = re; q.sq = se; }
             if (g.tx == TX - 1) { p.rho = re; p.sq = se; }
         }
+        double t[5];
+        {
+            double pp[5], qq[5];
+            load5(pp, s, g.uc + 2);
+            load5(qq, s, g.uc - 2);
+            if (g.mid_x) diss_terms<false>(t, qq, q.u, wz, p.u, pp, Cases{});
+            else diss_terms<true>(t, qq, q.u, wz, p.u, pp, cases_of(g.i0 + g.tx, P.nx));
+        }
         flux_dir<1>(acc, wz, vc, qsc, pc, p, q, C, 0);
-        double pp[5], qq[5];
-        load5(pp, s, g.uc + 2);
-        load5(qq, s, g.uc - 2);
-        if (g.mid_x) diss_dir<false>(acc, qq, q.u, wz, six, p.u, pp, C.dssp, g.cx);
-        else diss_dir<true>(acc, qq, q.u, wz, six, p.u, pp, C.dssp, g.cx);
+        diss_apply(acc, t, C.dssp);
     }
     // eta: rows j+-1 belong to other warps; evaluate their rho_i / square
     // from the u values loaded for the stencil.
@@ -397,14 +468,20 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, int k) {
         Nb p, q;
         load5(p.u, s, g.uc + UX);
         load5(q.u, s, g.uc - UX);
+        // rows j+-1 belong to other warps: evaluate their rho_i / square from
+        // the u values loaded for the stencil (no cross-warp dependency)
         aux_of(p.u[0], p.u[1], p.u[2], p.u[3], p.rho, p.sq);
         aux_of(q.u[0], q.u[1], q.u[2], q.u[3], q.rho, q.sq);
+        double t[5];
+        {
+            double pp[5], qq[5];
+            load5(pp, s, g.uc + 2 * UX);
+            load5(qq, s, g.uc - 2 * UX);
+            if (g.mid_y) diss_terms<false>(t, qq, q.u, wz, p.u, pp, Cases{});
+            else diss_terms<true>(t, qq, q.u, wz, p.u, pp, cases_of(g.j0 + g.ty, P.ny));
+        }
         flux_dir<2>(acc, wz, vc, qsc, pc, p, q, C, 1);
-        double pp[5], qq[5];
-        load5(pp, s, g.uc + 2 * UX);
-        load5(qq, s, g.uc - 2 * UX);
-        if (g.mid_y) diss_dir<false>(acc, qq, q.u, wz, six, p.u, pp, C.dssp, g.cy);
-        else diss_dir<true>(acc, qq, q.u, wz, six, p.u, pp, C.dssp, g.cy);
+        diss_apply(acc, t, C.dssp);
     }
     // zeta: everything from the register window (inter-iteration scalar
     // replacement along the sequential loop)
@@ -417,12 +494,13 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, int k) {
         }
         p.rho = g.ra[PI]; p.sq = g.sa[PI];
         q.rho = g.ra[Q]; q.sq = g.sa[Q];
-        flux_dir<3>(acc, wz, vc, qsc, pc, p, q, C, 2);
+        double t[5];
         if (is_mid(k, P.nz))
-            diss_dir<false>(acc, g.w[QQ], g.w[Q], wz, six, g.w[PI], g.w[PP], C.dssp, Cases{});
+            diss_terms<false>(t, g.w[QQ], g.w[Q], wz, g.w[PI], g.w[PP], Cases{});
         else
-            diss_dir<true>(acc, g.w[QQ], g.w[Q], wz, six, g.w[PI], g.w[PP], C.dssp,
-                           cases_of(k, P.nz));
+            diss_terms<true>(t, g.w[QQ], g.w[Q], wz, g.w[PI], g.w[PP], cases_of(k, P.nz));
+        flux_dir<3>(acc, wz, vc, qsc, pc, p, q, C, 2);
+        diss_apply(acc, t, C.dssp);
     }
     if (g.active) {
         const int o = g.ocol + P.sk * (k - P.k0);
@@ -434,14 +512,20 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, int k) {
     if (g.tx == 0) {
         const int slot = (int)(sq_k % STAGES);
         __threadfence_block();
-        const unsigned old = atomicAdd(&g.released[slot], 1u);
+        unsigned int *released = smem_released();
+        const unsigned old = atomicAdd(&released[slot], 1u);
         if (old == (unsigned)(TY - 1)) {
-            g.released[slot] = 0;
+            released[slot] = 0;
             __threadfence_block();
             const int kn = k + STAGES;
             if (kn <= g.kb + 1)
-                issue_plane(g.umap, g.fmap, P, const_cast<double *>(g.su), g.full, g.i0, g.j0, kn,
+                issue_plane(umap, fmap, P, su, smem_full(), g.i0, g.j0, kn,
                             kn < g.kb, sq_k + STAGES);
+#if SAFARA_L2PF > 0
+            if (kn + SAFARA_L2PF <= g.kb + 1)
+                prefetch_plane_l2(umap, fmap, P, g.i0, g.j0, kn + SAFARA_L2PF,
+                                  kn + SAFARA_L2PF < g.kb);
+#endif
         }
     }
 }
@@ -452,10 +536,9 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, int k) {
 // warp to release it).
 __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensorMap *fmap,
                                          const Params &P) {
-    extern __shared__ __align__(128) unsigned char smem_raw[];
-    double *su = reinterpret_cast<double *>(smem_raw);
-    uint64_t *full = reinterpret_cast<uint64_t *>(su + (size_t)STAGES * SLOT);
-    unsigned int *released = reinterpret_cast<unsigned int *>(full + STAGES);
+    double *su = smem_ring();
+    uint64_t *full = smem_full();
+    unsigned int *released = smem_released();
 
     const int tid = threadIdx.x;
 
@@ -470,35 +553,33 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensor
     }
     __syncthreads();
 
-    copy_faces(P);
-
     int ub = split_point((int)blockIdx.x, P.units, P.ncta);
     const int ue = split_point((int)blockIdx.x + 1, P.units, P.ncta);
 
+
     Seg g;
-    g.su = su;
-    g.full = full;
-    g.released = released;
-    g.umap = umap;
-    g.fmap = fmap;
     g.tx = tid % TX;
     g.ty = tid / TX;  // lane = tx, warp = ty
     g.seq0 = 0;
 
+    // The first segment's planes are requested before the boundary-face copy
+    // so that the copy overlaps their latency.
+    bool first = true;
+    if (ub < ue && tid == 0) {
+        int col, ka, kb;
+        segment_of(P, ub, ue, col, ka, kb);
+        const int nload = kb - ka + 2;
+        const int npre = nload < STAGES ? nload : STAGES;
+        const int i0 = 1 + (col % P.ntx) * TX, j0 = 1 + (col / P.ntx) * TY;
+        for (int s = 0; s < npre; ++s)
+            issue_plane(umap, fmap, P, su, full, i0, j0, ka + s, ka + s < kb, (uint32_t)s);
+    }
+    copy_faces(P);
+
     while (ub < ue) {
         // ---- segment: one column tile, a contiguous run of planes ----
-        int col, pidx, run;
-        decode_unit(P, ub, col, pidx, run);
-        {
-            const int left = min(run, ue - ub);
-            if (pidx < P.n0) {
-                g.ka = P.ka0 + pidx;
-                g.kb = min(P.kb0, g.ka + left);
-            } else {
-                g.ka = P.ka1 + (pidx - P.n0);
-                g.kb = min(P.kb1, g.ka + left);
-            }
-        }
+        int col;
+        segment_of(P, ub, ue, col, g.ka, g.kb);
         ub += g.kb - g.ka;
         const int ka = g.ka, kb = g.kb;
 
@@ -509,17 +590,16 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensor
         g.active = (i <= P.nx - 2) && (j <= P.ny - 2);
         const int nload = kb - ka + 2;  // planes ka .. kb+1
 
-        if (tid == 0) {
+        if (tid == 0 && !first) {
             const int npre = nload < STAGES ? nload : STAGES;
             for (int s = 0; s < npre; ++s)
                 issue_plane(umap, fmap, P, su, full, g.i0, g.j0, ka + s, ka + s < kb, g.seq0 + s);
         }
+        first = false;
 
         // Case flags (global indices, reading c12).
         g.mid_x = is_mid(g.i0, P.nx) && is_mid(g.i0 + TX - 1, P.nx);
         g.mid_y = is_mid(j, P.ny);
-        g.cx = cases_of(i, P.nx);
-        g.cy = cases_of(j, P.ny);
         g.uc = (g.ty + 2) * UX + (g.tx + HX);  // centre in the u tile
         g.ocol = i + P.sy * j;                  // own column offset (dim)
 
@@ -545,7 +625,7 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensor
         // One step body (instruction-cache footprint) and a register-move
         // rotation; unrolling by 5 for pure renaming measured slower (I$).
         for (int k = ka; k < kb; ++k) {
-            rhs_step<0>(g, P, k);
+            rhs_step<0>(g, P, umap, fmap, k);
 #pragma unroll
             for (int d = 0; d < 4; ++d) {
 #pragma unroll

@@ -16,7 +16,10 @@ constexpr int TX = 32;
 #endif
 constexpr int TY = SAFARA_TY;
 constexpr int NTHREADS = TX * TY;
-constexpr int STAGES = 5;            // u planes in the TMA ring
+#ifndef SAFARA_STAGES
+#define SAFARA_STAGES 4
+#endif
+constexpr int STAGES = SAFARA_STAGES;  // planes in the TMA ring
 // u tile: i halo of 2 plus one pad column each side.  The TMA box's first
 // element must be 16-byte aligned (fp64: even i), and tiles start at odd i
 // (interior begins at i = 1), so the box starts at i0 - 3 and is TX + 6 wide.
