@@ -36,6 +36,8 @@ def parse():
     ap.add_argument("--warmup", type=int, default=20)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="BT-C", help="BENCH-CLASS, e.g. BT-C, SP-B")
+    ap.add_argument("--grid", default=None,
+                    help="nx,ny,nz override (experiments only; dt of --config)")
     ap.add_argument("--strict", action="store_true", help="time the STRICT variant")
     ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -155,6 +157,13 @@ def config_of(args):
     return bench, cls, n, dt
 
 
+def grid_of(args, n):
+    if args.grid:
+        nx, ny, nz = (int(v) for v in args.grid.split(","))
+        return nx, ny, nz
+    return n, n, n
+
+
 def run_reference(args):
     """CPU oracle arm (rank 0 only)."""
     import nasgen
@@ -199,8 +208,11 @@ def run_single(args):
     torch.cuda.set_device(0)
     sr.init(0)
     bench, cls, n, dt = config_of(args)
-    inp = nasgen.make_class(bench, cls, seed=1)
-    nx = ny = nz = n
+    nx, ny, nz = grid_of(args, n)
+    if args.grid:
+        inp = nasgen.make_inputs(nx, ny, nz, seed=1, dt=dt, bench=bench, cls=cls)
+    else:
+        inp = nasgen.make_class(bench, cls, seed=1)
     c = sr.coeffs_nas(nx, ny, nz, dt)
     du, df = sr.pack(inp.u), sr.pack(inp.forcing)
     dr = torch.empty_like(du)
@@ -265,7 +277,8 @@ def run_single(args):
         "n_gpus": 1, "steps": args.steps, "warmup": args.warmup,
         "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "strong",
         "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-        "config": {"workload": nasgen.config_name(bench, cls), "grid": [nx, ny, nz],
+        "config": {"workload": nasgen.config_name(bench, cls) if not args.grid else
+                   f"{bench} compute_rhs {nx}x{ny}x{nz} fp64 (experiment grid)", "grid": [nx, ny, nz],
                    "points": pts, "variant": "strict" if args.strict else "production",
                    "l2": "inputs 3x176 MB > 126 MB L2, no flush", "parallelism": "single"},
         "hbm_gbs": achieved,

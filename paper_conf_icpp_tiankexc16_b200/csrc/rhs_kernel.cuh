@@ -395,6 +395,7 @@ __device__ __forceinline__ unsigned int *smem_released() {
 }
 
 struct Seg {
+    double *rptr;  // rhs of (i, j, k, m=0) for the current step
     int i0, j0, ka, kb, uc, ocol, tx, ty;
     bool in_grid, active, mid_x, mid_y;
     uint32_t seq0;
@@ -503,10 +504,16 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensor
         diss_apply(acc, t, C.dssp);
     }
     if (g.active) {
-        const int o = g.ocol + P.sk * (k - P.k0);
+        // rptr walks down the column one plane per step; the 5 component
+        // planes are sm apart (one 64-bit pointer instead of 5 addresses)
+        double *rp = g.rptr;
 #pragma unroll
-        for (int m = 0; m < 5; ++m) __stcs(P.r + o + P.sm * m, acc[m] * C.dt);
+        for (int m = 0; m < 5; ++m) {
+            __stcs(rp, acc[m] * C.dt);
+            rp += P.sm;
+        }
     }
+    g.rptr += P.sk;
     // release plane k's slot; the last warp out refills it with plane k+STAGES
     __syncwarp();
     if (g.tx == 0) {
@@ -602,6 +609,7 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensor
         g.mid_y = is_mid(j, P.ny);
         g.uc = (g.ty + 2) * UX + (g.tx + HX);  // centre in the u tile
         g.ocol = i + P.sy * j;                  // own column offset (dim)
+        g.rptr = P.r + (g.ocol + P.sk * (ka - P.k0));
 
         // Window at rotation 0: planes ka-2, ka-1 from global memory (read
         // once per segment), ka and ka+1 from the TMA ring.
