@@ -262,39 +262,54 @@ __device__ __forceinline__ void copy_faces(const Params &P) {
     const int full0 = has0 ? kl0 : kl1;  // first full plane; the second is always kl1
     const long long inner = (long long)(nx - 2) * (ny - 2);
     const long long total = nper + inner * nfull;
+    // Batches of FB points per thread: all 5*FB loads are in flight before
+    // the first store (one memory latency per batch, not per element).
+    constexpr int FB = 4;
     const long long stride = (long long)gridDim.x * blockDim.x;
-    for (long long t = (long long)blockIdx.x * blockDim.x + threadIdx.x; t < total; t += stride) {
-        int i, j, kl;
-        if (t < nper) {
-            kl = P.fk_lo + (int)(t / per);
-            int e = (int)(t % per);
-            if (e < nx) {
-                i = e; j = 0;
-            } else if (e < 2 * nx) {
-                i = e - nx; j = ny - 1;
-            } else {
-                e -= 2 * nx;
-                if (e < ny - 2) { i = 0; j = 1 + e; }
-                else { i = nx - 1; j = 1 + e - (ny - 2); }
-            }
-        } else {
-            const long long e = t - nper;
-            kl = (e < inner) ? full0 : kl1;
-            const int r = (int)(e % inner);
-            i = 1 + r % (nx - 2);
-            j = 1 + r / (nx - 2);
-        }
-        const int o = i + P.sy * j + P.sk * kl;
-        double v[5];  // all loads first: rhs may not alias forcing (ABI), but
-#pragma unroll    // the compiler cannot know that
-        for (int m = 0; m < 5; ++m) v[m] = __ldcs(P.f + o + P.sm * m);
+    for (long long t0 = (long long)blockIdx.x * blockDim.x + threadIdx.x; t0 < total;
+         t0 += stride * FB) {
+        int off[FB];
+        double v[FB][5];
 #pragma unroll
-        for (int m = 0; m < 5; ++m) __stcs(P.r + o + P.sm * m, v[m]);
+        for (int b = 0; b < FB; ++b) {
+            const long long t = t0 + (long long)b * stride;
+            off[b] = -1;
+            if (t < total) {
+                int i, j, kl;
+                const int ti = (int)t;  // faces < 2^31 points (validated extents)
+                if (t < nper) {
+                    kl = P.fk_lo + ti / per;
+                    int e = ti % per;
+                    if (e < nx) {
+                        i = e; j = 0;
+                    } else if (e < 2 * nx) {
+                        i = e - nx; j = ny - 1;
+                    } else {
+                        e -= 2 * nx;
+                        if (e < ny - 2) { i = 0; j = 1 + e; }
+                        else { i = nx - 1; j = 1 + e - (ny - 2); }
+                    }
+                } else {
+                    const int e = ti - (int)nper;
+                    kl = (e < inner) ? full0 : kl1;
+                    const int r = e % (int)inner;
+                    i = 1 + r % (nx - 2);
+                    j = 1 + r / (nx - 2);
+                }
+                off[b] = i + P.sy * j + P.sk * kl;
+#pragma unroll
+                for (int m = 0; m < 5; ++m) v[b][m] = __ldcs(P.f + off[b] + P.sm * m);
+            }
+        }
+#pragma unroll
+        for (int b = 0; b < FB; ++b)
+            if (off[b] >= 0) {
+#pragma unroll
+                for (int m = 0; m < 5; ++m) __stcs(P.r + off[b] + P.sm * m, v[b][m]);
+            }
     }
 }
 
-// Stage plane k: the u tile (halo 2 in i/j) and, for planes that are
-// computed, the forcing tile, both onto the slot's mbarrier.
 __device__ __forceinline__ void issue_plane(const CUtensorMap *umap, const CUtensorMap *fmap,
                                             const Params &P, double *su, uint64_t *full, int i0,
                                             int j0, int k, bool with_f, uint32_t seq) {
