@@ -39,7 +39,11 @@ def parse():
     ap.add_argument("--grid", default=None,
                     help="nx,ny,nz override (experiments only; dt of --config)")
     ap.add_argument("--strict", action="store_true", help="time the STRICT variant")
+    ap.add_argument("--dist", action="store_true",
+                    help="use the z-slab/NCCL path even on one rank (testing)")
     ap.add_argument("--e2e-steps", type=int, default=5)
+    ap.add_argument("--e2e-chunks", type=int, default=8,
+                    help="k-chunks of the pipelined H2D / compute / D2H e2e path")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--soak-s", type=float, default=1.0,
                     help="untimed passes before the timed region so the clock sampler "
@@ -261,12 +265,14 @@ def run_single(args):
     hu, hf = sr.pack(inp.u, pin=True), sr.pack(inp.forcing, pin=True)
     hr = torch.empty(hu.shape, dtype=torch.float64).pin_memory()
     for _ in range(2):
-        sr.rhs_host(hu, hf, hr, du, df, dr, nx, c, strict=args.strict, stream=stream)
+        sr.rhs_host(hu, hf, hr, du, df, dr, nx, c, strict=args.strict, nchunks=args.e2e_chunks,
+                    stream=stream)
     torch.cuda.synchronize()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     e0.record(stream)
     for _ in range(args.e2e_steps):
-        sr.rhs_host(hu, hf, hr, du, df, dr, nx, c, strict=args.strict, stream=stream)
+        sr.rhs_host(hu, hf, hr, du, df, dr, nx, c, strict=args.strict, nchunks=args.e2e_chunks,
+                    stream=stream)
     e1.record(stream)
     torch.cuda.synchronize()
     e2e_ms = e0.elapsed_time(e1) / args.e2e_steps
@@ -304,7 +310,7 @@ def main():
         run_reference(args)
         return
     world = int(os.environ.get("WORLD_SIZE", "1"))
-    if world > 1 or args.gpus > 1:
+    if world > 1 or args.gpus > 1 or args.dist:
         from paper_conf_icpp_tiankexc16_b200 import dist_bench
         dist_bench.run(args)
     else:

@@ -133,9 +133,13 @@ int safara_rhs_slab(const double *u_slab, const double *forcing_slab,
 
 /* End-to-end call with HOST arrays (canonical layout): copies u and forcing
  * host->device into the caller's device buffers u_dev/forcing_dev, runs the
- * pass into rhs_dev and copies rhs device->host, all asynchronously on
- * `stream` in `nchunks` k-chunks so that copies and compute overlap (host
- * buffers should be pinned).  The caller synchronises the stream.            */
+ * pass into rhs_dev and copies rhs device->host.  The grid is cut into
+ * `nchunks` k-chunks (>= 4 planes each, <= 64): H2D of chunk c+1, the kernel
+ * of chunk c and the D2H of chunk c-1 overlap (two internal copy streams,
+ * forked from and joined back into `stream`; host buffers must be pinned for
+ * the copies to be asynchronous).  One kernel launch per chunk.  Everything is
+ * ordered after prior work on `stream`, and work later enqueued on `stream`
+ * sees rhs_host complete.  The caller synchronises the stream.               */
 int safara_rhs_host(const double *u_host, const double *forcing_host,
                     double *rhs_host, double *u_dev, double *forcing_dev,
                     double *rhs_dev, int nx, int ny, int nz,

@@ -23,11 +23,17 @@ namespace {
 
 constexpr int kMaxDevices = 64;
 
+constexpr int kMaxChunks = 64;
+
 struct DeviceState {
     bool ready = false;
     int sms = 0;
     int ctas_fast = 0, ctas_strict = 0;
     cudaFuncAttributes attr_fast{}, attr_strict{};
+    // copy engines for safara_rhs_host's H2D / D2H pipeline (created at init)
+    cudaStream_t h2d = nullptr, d2h = nullptr;
+    cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+    cudaEvent_t ev_h[kMaxChunks] = {}, ev_c[kMaxChunks] = {};
 };
 
 DeviceState g_dev[kMaxDevices];
@@ -295,6 +301,14 @@ int safara_rhs_init(int device) {
     st.sms = sms;
     cudaError_t e = setup_rhs_fast(&st.ctas_fast, &st.attr_fast);
     if (e == cudaSuccess) e = setup_rhs_strict(&st.ctas_strict, &st.attr_strict);
+    if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&st.h2d, cudaStreamNonBlocking);
+    if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&st.d2h, cudaStreamNonBlocking);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&st.ev_fork, cudaEventDisableTiming);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&st.ev_join, cudaEventDisableTiming);
+    for (int c = 0; c < kMaxChunks && e == cudaSuccess; ++c) {
+        e = cudaEventCreateWithFlags(&st.ev_h[c], cudaEventDisableTiming);
+        if (e == cudaSuccess) e = cudaEventCreateWithFlags(&st.ev_c[c], cudaEventDisableTiming);
+    }
     cudaSetDevice(prev);
     if (e != cudaSuccess) return SAFARA_ERR_CUDA;
     st.ready = true;
@@ -367,21 +381,53 @@ int safara_rhs_slab(const double *u_slab, const double *forcing_slab, double *rh
 int safara_rhs_host(const double *u_host, const double *forcing_host, double *rhs_host,
                     double *u_dev, double *forcing_dev, double *rhs_dev, int nx, int ny, int nz,
                     const safara_coeffs_t *coeffs, int flags, int nchunks, void *stream) {
-    (void)nchunks;
     if (!u_host || !forcing_host || !rhs_host) return SAFARA_ERR_ARG;
     safara_dims_t d;
     int rc = safara_dims_canonical(nx, ny, nz, &d);
     if (rc) return rc;
-    const size_t bytes = (size_t)d.sk * nz * sizeof(double);
-    cudaStream_t s = (cudaStream_t)stream;
-    if (cudaMemcpyAsync(u_dev, u_host, bytes, cudaMemcpyHostToDevice, s) != cudaSuccess ||
-        cudaMemcpyAsync(forcing_dev, forcing_host, bytes, cudaMemcpyHostToDevice, s) != cudaSuccess)
-        return SAFARA_ERR_CUDA;
-    rc = safara_rhs_ex(u_dev, forcing_dev, rhs_dev, &d, coeffs, flags, stream);
+    rc = validate(&d, nz);
     if (rc) return rc;
-    if (cudaMemcpyAsync(rhs_host, rhs_dev, bytes, cudaMemcpyDeviceToHost, s) != cudaSuccess)
-        return SAFARA_ERR_CUDA;
-    return SAFARA_OK;
+    const long long bytes = (long long)d.sk * nz * (long long)sizeof(double);
+    rc = check_ptrs(u_dev, bytes, forcing_dev, bytes, rhs_dev, bytes);
+    if (rc) return rc;
+    int dev;
+    rc = current_device(&dev);
+    if (rc) return rc;
+    DeviceState &st = g_dev[dev];
+    std::lock_guard<std::mutex> lock(g_mutex);  // the copy streams/events are per device
+    cudaStream_t s = (cudaStream_t)stream;
+    // k-chunks of >= 4 planes; chunk c computes planes [z_c, z_{c+1}) once the
+    // H2D of chunk c+1 (which holds its +2 ghost planes) has landed, and its
+    // rhs planes go back while later chunks are copied in and computed.
+    int C = std::max(1, std::min(std::min(nchunks, kMaxChunks), nz / 4));
+    auto z = [&](int c) { return (int)((long long)nz * c / C); };
+    const size_t plane = (size_t)d.sk * sizeof(double);
+    bool ok = cudaEventRecord(st.ev_fork, s) == cudaSuccess &&
+              cudaStreamWaitEvent(st.h2d, st.ev_fork, 0) == cudaSuccess &&
+              cudaStreamWaitEvent(st.d2h, st.ev_fork, 0) == cudaSuccess;
+    for (int c = 0; ok && c < C; ++c) {
+        const size_t off = (size_t)z(c) * d.sk, len = (size_t)(z(c + 1) - z(c)) * plane;
+        ok = cudaMemcpyAsync(u_dev + off, u_host + off, len, cudaMemcpyHostToDevice, st.h2d) ==
+                 cudaSuccess &&
+             cudaMemcpyAsync(forcing_dev + off, forcing_host + off, len, cudaMemcpyHostToDevice,
+                             st.h2d) == cudaSuccess &&
+             cudaEventRecord(st.ev_h[c], st.h2d) == cudaSuccess;
+    }
+    for (int c = 0; ok && c < C; ++c) {
+        ok = cudaStreamWaitEvent(s, st.ev_h[std::min(c + 1, C - 1)], 0) == cudaSuccess;
+        if (!ok) break;
+        rc = launch(u_dev, forcing_dev, rhs_dev, d, nz, nz, 0, 0, std::max(z(c), 1),
+                    std::min(z(c + 1), nz - 1), 0, 0, z(c), z(c + 1), coeffs, flags, s);
+        if (rc) return rc;
+        const size_t off = (size_t)z(c) * d.sk, len = (size_t)(z(c + 1) - z(c)) * plane;
+        ok = cudaEventRecord(st.ev_c[c], s) == cudaSuccess &&
+             cudaStreamWaitEvent(st.d2h, st.ev_c[c], 0) == cudaSuccess &&
+             cudaMemcpyAsync(rhs_host + off, rhs_dev + off, len, cudaMemcpyDeviceToHost,
+                             st.d2h) == cudaSuccess;
+    }
+    ok = ok && cudaEventRecord(st.ev_join, st.d2h) == cudaSuccess &&
+         cudaStreamWaitEvent(s, st.ev_join, 0) == cudaSuccess;
+    return ok ? SAFARA_OK : SAFARA_ERR_CUDA;
 }
 
 int64_t safara_launch_count(void) { return g_launches.load(); }

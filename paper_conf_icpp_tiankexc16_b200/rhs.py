@@ -121,7 +121,7 @@ def rhs_slab(u_slab: torch.Tensor, forcing_slab: torch.Tensor, out_slab: torch.T
 
 def rhs_host(u_host: torch.Tensor, f_host: torch.Tensor, r_host: torch.Tensor,
              u_dev: torch.Tensor, f_dev: torch.Tensor, r_dev: torch.Tensor, nx: int,
-             coeffs: Coeffs, strict: bool = False, nchunks: int = 1, stream=None):
+             coeffs: Coeffs, strict: bool = False, nchunks: int = 8, stream=None):
     """End-to-end pass on host (pinned) canonical tensors through device buffers."""
     nz, _, ny, _ = u_host.shape
     flags = SAFARA_FLAG_STRICT if strict else 0

@@ -158,15 +158,18 @@ def test_slab_decomposition(nz, p, split, strict):
         assert_tol(a, oracle_rhs(inp))
 
 
-def test_host_e2e_path():
+@pytest.mark.parametrize("nchunks", [1, 3, 8])
+def test_host_e2e_path(nchunks):
     inp = nasgen.make_class("SP", "W", seed=6)
     nz, ny, nx, _ = inp.u.shape
     hu, hf = sr.pack(inp.u, pin=True), sr.pack(inp.forcing, pin=True)
     hr = torch.zeros_like(hu).pin_memory()
     du, df, dr = (torch.empty(hu.shape, dtype=torch.float64, device="cuda") for _ in range(3))
     c = sr.coeffs_nas(nx, ny, nz, inp.dt)
-    sr.rhs_host(hu, hf, hr, du, df, dr, nx, c, strict=True)
+    n0 = sr.launch_count()
+    sr.rhs_host(hu, hf, hr, du, df, dr, nx, c, strict=True, nchunks=nchunks)
     torch.cuda.synchronize()
+    assert sr.launch_count() - n0 == min(nchunks, nz // 4)
     assert np.array_equal(sr.unpack(hr, nx), oracle_rhs(inp))
 
 
