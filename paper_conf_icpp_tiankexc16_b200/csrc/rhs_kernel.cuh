@@ -33,6 +33,21 @@
 
 #include "safara_internal.h"
 
+// Production variant: number of independent partial sums the three
+// directions accumulate into (1 = the NAS chain; STRICT always uses 1).
+#if SAFARA_STRICT_BUILD
+#undef SAFARA_PSUMS
+#define SAFARA_PSUMS 1
+#undef SAFARA_ZETA_FIRST
+#define SAFARA_ZETA_FIRST 1
+#elif !defined(SAFARA_PSUMS)
+#define SAFARA_PSUMS 2
+#endif
+// production: form the zeta (register-only) partial sum first, while the
+// xi/eta shared-memory loads are in flight (needs PSUMS >= 2)
+#ifndef SAFARA_ZETA_FIRST
+#define SAFARA_ZETA_FIRST 1
+#endif
 #ifndef SAFARA_L2PF
 #define SAFARA_L2PF 0  // planes beyond the ring to prefetch into L2 (0 = off)
 #endif
@@ -157,7 +172,17 @@ __device__ __forceinline__ void load5(double (&a)[5], const double *su, int uidx
 
 // Flux differences along one axis (App. A steps 2 / 4 / 6).  MOM = index of
 // the momentum component along the axis (1 = xi, 2 = eta, 3 = zeta).
-template <int MOM>
+// `acc[m] = acc[m] + x`, or `acc[m] = x` for the first term of an independent
+// partial sum (INIT): the production variant accumulates the directions in
+// separate partial sums (shorter dependency chains; every stencil difference
+// is still formed exactly in NAS order, reading c6).
+template <bool INIT>
+__device__ __forceinline__ double acc_add(double a, double x) {
+    if (INIT) return x;
+    return a + x;
+}
+
+template <int MOM, bool INIT = false>
 __device__ __forceinline__ void flux_dir(double (&acc)[5], const double (&cu)[5],
                                          const double (&vc)[3], double qsc, double pc,
                                          const Nb &p, const Nb &q, const Coef &C, int ax) {
@@ -170,11 +195,11 @@ __device__ __forceinline__ void flux_dir(double (&acc)[5], const double (&cu)[5]
     const double wp = vp[MOM - 1], wq = vq[MOM - 1], wc = vc[MOM - 1];
     const double t2 = C.t2[ax];
 
-    acc[0] = acc[0] + C.d1[ax][0] * d2(p.u[0], cu[0], q.u[0]);
+    acc[0] = acc_add<INIT>(acc[0], C.d1[ax][0] * d2(p.u[0], cu[0], q.u[0]));
     acc[0] = acc[0] - t2 * (p.u[MOM] - q.u[MOM]);
 #pragma unroll
     for (int m = 1; m <= 3; ++m) {
-        acc[m] = acc[m] + C.d1[ax][m] * d2(p.u[m], cu[m], q.u[m]);
+        acc[m] = acc_add<INIT>(acc[m], C.d1[ax][m] * d2(p.u[m], cu[m], q.u[m]));
         if (m == MOM) {
             acc[m] = acc[m] + C.con2x43[ax] * d2(wp, wc, wq);
             acc[m] = acc[m] - t2 * ((p.u[m] * wp - q.u[m] * wq) +
@@ -184,7 +209,7 @@ __device__ __forceinline__ void flux_dir(double (&acc)[5], const double (&cu)[5]
             acc[m] = acc[m] - t2 * (p.u[m] * wp - q.u[m] * wq);
         }
     }
-    acc[4] = acc[4] + C.d1[ax][4] * d2(p.u[4], cu[4], q.u[4]);
+    acc[4] = acc_add<INIT>(acc[4], C.d1[ax][4] * d2(p.u[4], cu[4], q.u[4]));
     acc[4] = acc[4] + C.con3[ax] * d2(p.sq * p.rho, qsc, q.sq * q.rho);
     acc[4] = acc[4] + C.con4[ax] * d2(wp * wp, wc * wc, wq * wq);
     acc[4] = acc[4] + C.con5[ax] * d2(p.u[4] * p.rho, pc, q.u[4] * q.rho);
@@ -431,6 +456,12 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensor
     // forcing(k): staged by the same TMA as plane k (reuse count 1, so it only
     // needs latency hiding, not a register slot)
     double acc[5];
+#if SAFARA_PSUMS >= 2
+    double acc_z[5];
+#endif
+#if SAFARA_PSUMS >= 3
+    double acc_y[5];
+#endif
     {
         const double *fs = s + U_SLOT;
 #pragma unroll
@@ -449,6 +480,31 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensor
     vc[2] = wz[3] * r0;
     const double qsc = s0 * r0;
     const double pc = wz[4] * r0;
+#if SAFARA_ZETA_FIRST
+    // zeta: everything from the register window (inter-iteration scalar
+    // replacement along the sequential loop)
+    {
+        Nb p, q;
+#pragma unroll
+        for (int m = 0; m < 5; ++m) {
+            p.u[m] = g.w[PI][m];
+            q.u[m] = g.w[Q][m];
+        }
+        p.rho = g.ra[PI]; p.sq = g.sa[PI];
+        q.rho = g.ra[Q]; q.sq = g.sa[Q];
+        double t[5];
+        if (is_mid(k, P.nz))
+            diss_terms<false>(t, g.w[QQ], g.w[Q], wz, g.w[PI], g.w[PP], Cases{});
+        else
+            diss_terms<true>(t, g.w[QQ], g.w[Q], wz, g.w[PI], g.w[PP], cases_of(k, P.nz));
+#if SAFARA_PSUMS >= 2
+        flux_dir<3, true>(acc_z, wz, vc, qsc, pc, p, q, C, 2);
+        diss_apply(acc_z, t, C.dssp);
+#else
+        flux_dir<3>(acc, wz, vc, qsc, pc, p, q, C, 2);
+        diss_apply(acc, t, C.dssp);
+#endif
+    }
     // xi: rho_i/square of i+-1 are the neighbour lanes' own values; lanes 0
     // and 31 evaluate their outside neighbour themselves.
     {
@@ -496,8 +552,69 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensor
             if (g.mid_y) diss_terms<false>(t, qq, q.u, wz, p.u, pp, Cases{});
             else diss_terms<true>(t, qq, q.u, wz, p.u, pp, cases_of(g.j0 + g.ty, P.ny));
         }
+#if SAFARA_PSUMS >= 3
+        flux_dir<2, true>(acc_y, wz, vc, qsc, pc, p, q, C, 1);
+        diss_apply(acc_y, t, C.dssp);
+#else
         flux_dir<2>(acc, wz, vc, qsc, pc, p, q, C, 1);
         diss_apply(acc, t, C.dssp);
+#endif
+    }
+#else
+    // xi: rho_i/square of i+-1 are the neighbour lanes' own values; lanes 0
+    // and 31 evaluate their outside neighbour themselves.
+    {
+        Nb p, q;
+        load5(p.u, s, g.uc + 1);
+        load5(q.u, s, g.uc - 1);
+        p.rho = __shfl_down_sync(FULL, r0, 1);
+        p.sq = __shfl_down_sync(FULL, s0, 1);
+        q.rho = __shfl_up_sync(FULL, r0, 1);
+        q.sq = __shfl_up_sync(FULL, s0, 1);
+        {
+            const bool left = (g.tx == 0);
+            double re, se;
+            aux_of(left ? q.u[0] : p.u[0], left ? q.u[1] : p.u[1], left ? q.u[2] : p.u[2],
+                   left ? q.u[3] : p.u[3], re, se);
+            if (left) { q.rho = re; q.sq = se; }
+            if (g.tx == TX - 1) { p.rho = re; p.sq = se; }
+        }
+        double t[5];
+        {
+            double pp[5], qq[5];
+            load5(pp, s, g.uc + 2);
+            load5(qq, s, g.uc - 2);
+            if (g.mid_x) diss_terms<false>(t, qq, q.u, wz, p.u, pp, Cases{});
+            else diss_terms<true>(t, qq, q.u, wz, p.u, pp, cases_of(g.i0 + g.tx, P.nx));
+        }
+        flux_dir<1>(acc, wz, vc, qsc, pc, p, q, C, 0);
+        diss_apply(acc, t, C.dssp);
+    }
+    // eta: rows j+-1 belong to other warps; evaluate their rho_i / square
+    // from the u values loaded for the stencil.
+    {
+        Nb p, q;
+        load5(p.u, s, g.uc + UX);
+        load5(q.u, s, g.uc - UX);
+        // rows j+-1 belong to other warps: evaluate their rho_i / square from
+        // the u values loaded for the stencil (no cross-warp dependency)
+        aux_of(p.u[0], p.u[1], p.u[2], p.u[3], p.rho, p.sq);
+        aux_of(q.u[0], q.u[1], q.u[2], q.u[3], q.rho, q.sq);
+        double t[5];
+        {
+            double pp[5], qq[5];
+            load5(pp, s, g.uc + 2 * UX);
+            load5(qq, s, g.uc - 2 * UX);
+            if (g.mid_y) diss_terms<false>(t, qq, q.u, wz, p.u, pp, Cases{});
+            else diss_terms<true>(t, qq, q.u, wz, p.u, pp, cases_of(g.j0 + g.ty, P.ny));
+        }
+#if SAFARA_PSUMS >= 3
+        flux_dir<2, true>(acc_y, wz, vc, qsc, pc, p, q, C, 1);
+        diss_apply(acc_y, t, C.dssp);
+#else
+        flux_dir<2>(acc, wz, vc, qsc, pc, p, q, C, 1);
+        diss_apply(acc, t, C.dssp);
+#endif
     }
     // zeta: everything from the register window (inter-iteration scalar
     // replacement along the sequential loop)
@@ -515,9 +632,22 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensor
             diss_terms<false>(t, g.w[QQ], g.w[Q], wz, g.w[PI], g.w[PP], Cases{});
         else
             diss_terms<true>(t, g.w[QQ], g.w[Q], wz, g.w[PI], g.w[PP], cases_of(k, P.nz));
+#if SAFARA_PSUMS >= 2
+        flux_dir<3, true>(acc_z, wz, vc, qsc, pc, p, q, C, 2);
+        diss_apply(acc_z, t, C.dssp);
+#else
         flux_dir<3>(acc, wz, vc, qsc, pc, p, q, C, 2);
         diss_apply(acc, t, C.dssp);
+#endif
     }
+#endif
+#if SAFARA_PSUMS == 2
+#pragma unroll
+    for (int m = 0; m < 5; ++m) acc[m] = acc[m] + acc_z[m];
+#elif SAFARA_PSUMS == 3
+#pragma unroll
+    for (int m = 0; m < 5; ++m) acc[m] = acc[m] + (acc_y[m] + acc_z[m]);
+#endif
     if (g.active) {
         // rptr walks down the column one plane per step; the 5 component
         // planes are sm apart (one 64-bit pointer instead of 5 addresses)
