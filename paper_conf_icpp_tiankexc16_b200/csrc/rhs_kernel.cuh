@@ -35,18 +35,24 @@
 
 // Production variant: number of independent partial sums the three
 // directions accumulate into (1 = the NAS chain; STRICT always uses 1).
+// Production only: form the zeta (register-only) partial sum first, while
+// the xi/eta shared-memory loads are in flight (needs PSUMS >= 2).  STRICT
+// keeps the NAS accumulation order forcing, xi, eta, zeta.
 #if SAFARA_STRICT_BUILD
 #undef SAFARA_PSUMS
 #define SAFARA_PSUMS 1
 #undef SAFARA_ZETA_FIRST
-#define SAFARA_ZETA_FIRST 1
-#elif !defined(SAFARA_PSUMS)
+#define SAFARA_ZETA_FIRST 0
+#else
+#ifndef SAFARA_PSUMS
 #define SAFARA_PSUMS 2
 #endif
-// production: form the zeta (register-only) partial sum first, while the
-// xi/eta shared-memory loads are in flight (needs PSUMS >= 2)
 #ifndef SAFARA_ZETA_FIRST
 #define SAFARA_ZETA_FIRST 1
+#endif
+#endif
+#if SAFARA_ZETA_FIRST && SAFARA_PSUMS < 2
+#error "SAFARA_ZETA_FIRST reorders the accumulation: it needs SAFARA_PSUMS >= 2"
 #endif
 #ifndef SAFARA_L2PF
 #define SAFARA_L2PF 0  // planes beyond the ring to prefetch into L2 (0 = off)
