@@ -211,6 +211,9 @@ int launch(const double *u, const double *f, double *r, const safara_dims_t &d, 
         ncta = std::min<long long>(max_ctas, 16);
     }
     p.ncta = (int)ncta;
+    // SMs the compute grid leaves idle take the boundary faces
+    p.nface_cta = (fk_hi > fk_lo && p.units > 0 && ncta < max_ctas)
+                      ? (int)std::min<long long>(max_ctas - ncta, 32) : 0;
 
     CUtensorMap umap, fmap;
     int pj, pm, pk;

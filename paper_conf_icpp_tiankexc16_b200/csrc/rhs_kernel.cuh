@@ -279,7 +279,7 @@ __device__ __forceinline__ void diss_apply(double (&acc)[5], const double (&t)[5
 
 // Copy forcing -> rhs on this launch's boundary-face points (rhs = forcing,
 // unscaled; App. A step 1, reading c3), spread over all CTAs.
-__device__ __forceinline__ void copy_faces(const Params &P) {
+__device__ __forceinline__ void copy_faces(const Params &P, int cta, int nctas) {
     const int nx = P.nx, ny = P.ny;
     const int per = 2 * nx + 2 * (ny - 2);
     const int nloc = P.fk_hi - P.fk_lo;
@@ -296,8 +296,8 @@ __device__ __forceinline__ void copy_faces(const Params &P) {
     // Batches of FB points per thread: all 5*FB loads are in flight before
     // the first store (one memory latency per batch, not per element).
     constexpr int FB = 4;
-    const long long stride = (long long)gridDim.x * blockDim.x;
-    for (long long t0 = (long long)blockIdx.x * blockDim.x + threadIdx.x; t0 < total;
+    const long long stride = (long long)nctas * blockDim.x;
+    for (long long t0 = (long long)cta * blockDim.x + threadIdx.x; t0 < total;
          t0 += stride * FB) {
         int off[FB];
         double v[FB][5];
@@ -694,6 +694,12 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensor
 // warp to release it).
 __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensorMap *fmap,
                                          const Params &P) {
+    // Extra CTAs beyond the compute grid (on SMs the lockstep schedule leaves
+    // idle) only copy the boundary faces.
+    if ((int)blockIdx.x >= P.ncta) {
+        copy_faces(P, (int)blockIdx.x - P.ncta, P.nface_cta);
+        return;
+    }
     double *su = smem_ring();
     uint64_t *full = smem_full();
     unsigned int *released = smem_released();
@@ -732,7 +738,7 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensor
         for (int s = 0; s < npre; ++s)
             issue_plane(umap, fmap, P, su, full, i0, j0, ka + s, ka + s < kb, (uint32_t)s);
     }
-    copy_faces(P);
+    if (P.nface_cta == 0) copy_faces(P, (int)blockIdx.x, P.ncta);
 
     while (ub < ue) {
         // ---- segment: one column tile, a contiguous run of planes ----

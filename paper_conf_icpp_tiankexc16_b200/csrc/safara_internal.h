@@ -58,7 +58,8 @@ struct Params {
     int ntx, nty;          // column tiles
     int ncol;              // ntx * nty
     int chunk;             // planes per chunk of the chunk-major unit order
-    int ncta;              // CTAs in the grid
+    int ncta;              // compute CTAs (the grid has ncta + nface_cta)
+    int nface_cta;         // extra CTAs that only copy boundary faces (0: compute CTAs do it)
     int units;             // ncol*nplanes (column-plane work items, < 2^31)
     int fk_lo, fk_hi;      // local planes whose boundary faces this launch copies
     int pos_j, pos_m, pos_k;  // tensor-map dimension holding j, m, k
