@@ -461,6 +461,7 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensor
 
     // forcing(k): staged by the same TMA as plane k (reuse count 1, so it only
     // needs latency hiding, not a register slot)
+    unsigned rel_old = 0;  // slot-release counter value seen by lane 0
     double acc[5];
 #if SAFARA_PSUMS >= 2
     double acc_z[5];
@@ -558,6 +559,13 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensor
             if (g.mid_y) diss_terms<false>(t, qq, q.u, wz, p.u, pp, Cases{});
             else diss_terms<true>(t, qq, q.u, wz, p.u, pp, cases_of(g.j0 + g.ty, P.ny));
         }
+        // Every read of plane k's slot is done: release it now, act on the
+        // counter at the end of the step (its latency hides behind eta).
+        __syncwarp();
+        if (g.tx == 0) {
+            __threadfence_block();
+            rel_old = atomicAdd(&smem_released()[(int)(sq_k % STAGES)], 1u);
+        }
 #if SAFARA_PSUMS >= 3
         flux_dir<2, true>(acc_y, wz, vc, qsc, pc, p, q, C, 1);
         diss_apply(acc_y, t, C.dssp);
@@ -614,6 +622,13 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensor
             if (g.mid_y) diss_terms<false>(t, qq, q.u, wz, p.u, pp, Cases{});
             else diss_terms<true>(t, qq, q.u, wz, p.u, pp, cases_of(g.j0 + g.ty, P.ny));
         }
+        // Every read of plane k's slot is done: release it now, act on the
+        // counter at the end of the step (its latency hides behind eta).
+        __syncwarp();
+        if (g.tx == 0) {
+            __threadfence_block();
+            rel_old = atomicAdd(&smem_released()[(int)(sq_k % STAGES)], 1u);
+        }
 #if SAFARA_PSUMS >= 3
         flux_dir<2, true>(acc_y, wz, vc, qsc, pc, p, q, C, 1);
         diss_apply(acc_y, t, C.dssp);
@@ -665,26 +680,19 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensor
         }
     }
     g.rptr += P.sk;
-    // release plane k's slot; the last warp out refills it with plane k+STAGES
-    __syncwarp();
-    if (g.tx == 0) {
-        const int slot = (int)(sq_k % STAGES);
+    // the last warp out of plane k (see the release above) refills its slot
+    if (g.tx == 0 && rel_old == (unsigned)(TY - 1)) {
+        smem_released()[(int)(sq_k % STAGES)] = 0;
         __threadfence_block();
-        unsigned int *released = smem_released();
-        const unsigned old = atomicAdd(&released[slot], 1u);
-        if (old == (unsigned)(TY - 1)) {
-            released[slot] = 0;
-            __threadfence_block();
-            const int kn = k + STAGES;
-            if (kn <= g.kb + 1)
-                issue_plane(umap, fmap, P, su, smem_full(), g.i0, g.j0, kn,
-                            kn < g.kb, sq_k + STAGES);
+        const int kn = k + STAGES;
+        if (kn <= g.kb + 1)
+            issue_plane(umap, fmap, P, su, smem_full(), g.i0, g.j0, kn, kn < g.kb,
+                        sq_k + STAGES);
 #if SAFARA_L2PF > 0
-            if (kn + SAFARA_L2PF <= g.kb + 1)
-                prefetch_plane_l2(umap, fmap, P, g.i0, g.j0, kn + SAFARA_L2PF,
-                                  kn + SAFARA_L2PF < g.kb);
+        if (kn + SAFARA_L2PF <= g.kb + 1)
+            prefetch_plane_l2(umap, fmap, P, g.i0, g.j0, kn + SAFARA_L2PF,
+                              kn + SAFARA_L2PF < g.kb);
 #endif
-        }
     }
 }
 
