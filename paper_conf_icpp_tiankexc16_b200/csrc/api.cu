@@ -221,8 +221,11 @@ int launch(const double *u, const double *f, double *r, const safara_dims_t &d, 
     if (rc) return rc;
     rc = encode_map(&fmap, f, d, nzf, FX, TY, &pj, &pm, &pk);
     if (rc) return rc;
-    cudaError_t e = strict ? launch_rhs_strict(umap, fmap, p, stream)
-                           : launch_rhs_fast(umap, fmap, p, stream);
+    bool ud = true;
+    for (int ax = 0; ax < 3; ++ax)
+        for (int m = 1; m < 5; ++m) ud = ud && (p.c.d1[ax][m] == p.c.d1[ax][0]);
+    cudaError_t e = strict ? launch_rhs_strict(umap, fmap, p, ud, stream)
+                           : launch_rhs_fast(umap, fmap, p, ud, stream);
     if (e != cudaSuccess) return SAFARA_ERR_CUDA;
     g_launches.fetch_add(1, std::memory_order_relaxed);
     return SAFARA_OK;

@@ -188,7 +188,7 @@ __device__ __forceinline__ double acc_add(double a, double x) {
     return a + x;
 }
 
-template <int MOM, bool INIT = false>
+template <int MOM, bool INIT, bool UD>
 __device__ __forceinline__ void flux_dir(double (&acc)[5], const double (&cu)[5],
                                          const double (&vc)[3], double qsc, double pc,
                                          const Nb &p, const Nb &q, const Coef &C, int ax) {
@@ -205,7 +205,7 @@ __device__ __forceinline__ void flux_dir(double (&acc)[5], const double (&cu)[5]
     acc[0] = acc[0] - t2 * (p.u[MOM] - q.u[MOM]);
 #pragma unroll
     for (int m = 1; m <= 3; ++m) {
-        acc[m] = acc_add<INIT>(acc[m], C.d1[ax][m] * d2(p.u[m], cu[m], q.u[m]));
+        acc[m] = acc_add<INIT>(acc[m], C.d1[ax][UD ? 0 : m] * d2(p.u[m], cu[m], q.u[m]));
         if (m == MOM) {
             acc[m] = acc[m] + C.con2x43[ax] * d2(wp, wc, wq);
             acc[m] = acc[m] - t2 * ((p.u[m] * wp - q.u[m] * wq) +
@@ -215,7 +215,7 @@ __device__ __forceinline__ void flux_dir(double (&acc)[5], const double (&cu)[5]
             acc[m] = acc[m] - t2 * (p.u[m] * wp - q.u[m] * wq);
         }
     }
-    acc[4] = acc_add<INIT>(acc[4], C.d1[ax][4] * d2(p.u[4], cu[4], q.u[4]));
+    acc[4] = acc_add<INIT>(acc[4], C.d1[ax][UD ? 0 : 4] * d2(p.u[4], cu[4], q.u[4]));
     acc[4] = acc[4] + C.con3[ax] * d2(p.sq * p.rho, qsc, q.sq * q.rho);
     acc[4] = acc[4] + C.con4[ax] * d2(wp * wp, wc * wc, wq * wq);
     acc[4] = acc[4] + C.con5[ax] * d2(p.u[4] * p.rho, pc, q.u[4] * q.rho);
@@ -449,7 +449,7 @@ struct Seg {
     double ra[5], sa[5];
 };
 
-template <int R>
+template <int R, bool UD>
 __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensorMap *umap,
                                          const CUtensorMap *fmap, int k) {
     constexpr int QQ = R % 5, Q = (R + 1) % 5, Z = (R + 2) % 5, PI = (R + 3) % 5, PP = (R + 4) % 5;
@@ -505,10 +505,10 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensor
         else
             diss_terms<true>(t, g.w[QQ], g.w[Q], wz, g.w[PI], g.w[PP], cases_of(k, P.nz));
 #if SAFARA_PSUMS >= 2
-        flux_dir<3, true>(acc_z, wz, vc, qsc, pc, p, q, C, 2);
+        flux_dir<3, true, UD>(acc_z, wz, vc, qsc, pc, p, q, C, 2);
         diss_apply(acc_z, t, C.dssp);
 #else
-        flux_dir<3>(acc, wz, vc, qsc, pc, p, q, C, 2);
+        flux_dir<3, false, UD>(acc, wz, vc, qsc, pc, p, q, C, 2);
         diss_apply(acc, t, C.dssp);
 #endif
     }
@@ -538,7 +538,7 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensor
             if (g.mid_x) diss_terms<false>(t, qq, q.u, wz, p.u, pp, Cases{});
             else diss_terms<true>(t, qq, q.u, wz, p.u, pp, cases_of(g.i0 + g.tx, P.nx));
         }
-        flux_dir<1>(acc, wz, vc, qsc, pc, p, q, C, 0);
+        flux_dir<1, false, UD>(acc, wz, vc, qsc, pc, p, q, C, 0);
         diss_apply(acc, t, C.dssp);
     }
     // eta: rows j+-1 belong to other warps; evaluate their rho_i / square
@@ -567,10 +567,10 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensor
             rel_old = atomicAdd(&smem_released()[(int)(sq_k % STAGES)], 1u);
         }
 #if SAFARA_PSUMS >= 3
-        flux_dir<2, true>(acc_y, wz, vc, qsc, pc, p, q, C, 1);
+        flux_dir<2, true, UD>(acc_y, wz, vc, qsc, pc, p, q, C, 1);
         diss_apply(acc_y, t, C.dssp);
 #else
-        flux_dir<2>(acc, wz, vc, qsc, pc, p, q, C, 1);
+        flux_dir<2, false, UD>(acc, wz, vc, qsc, pc, p, q, C, 1);
         diss_apply(acc, t, C.dssp);
 #endif
     }
@@ -601,7 +601,7 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensor
             if (g.mid_x) diss_terms<false>(t, qq, q.u, wz, p.u, pp, Cases{});
             else diss_terms<true>(t, qq, q.u, wz, p.u, pp, cases_of(g.i0 + g.tx, P.nx));
         }
-        flux_dir<1>(acc, wz, vc, qsc, pc, p, q, C, 0);
+        flux_dir<1, false, UD>(acc, wz, vc, qsc, pc, p, q, C, 0);
         diss_apply(acc, t, C.dssp);
     }
     // eta: rows j+-1 belong to other warps; evaluate their rho_i / square
@@ -630,10 +630,10 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensor
             rel_old = atomicAdd(&smem_released()[(int)(sq_k % STAGES)], 1u);
         }
 #if SAFARA_PSUMS >= 3
-        flux_dir<2, true>(acc_y, wz, vc, qsc, pc, p, q, C, 1);
+        flux_dir<2, true, UD>(acc_y, wz, vc, qsc, pc, p, q, C, 1);
         diss_apply(acc_y, t, C.dssp);
 #else
-        flux_dir<2>(acc, wz, vc, qsc, pc, p, q, C, 1);
+        flux_dir<2, false, UD>(acc, wz, vc, qsc, pc, p, q, C, 1);
         diss_apply(acc, t, C.dssp);
 #endif
     }
@@ -654,10 +654,10 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensor
         else
             diss_terms<true>(t, g.w[QQ], g.w[Q], wz, g.w[PI], g.w[PP], cases_of(k, P.nz));
 #if SAFARA_PSUMS >= 2
-        flux_dir<3, true>(acc_z, wz, vc, qsc, pc, p, q, C, 2);
+        flux_dir<3, true, UD>(acc_z, wz, vc, qsc, pc, p, q, C, 2);
         diss_apply(acc_z, t, C.dssp);
 #else
-        flux_dir<3>(acc, wz, vc, qsc, pc, p, q, C, 2);
+        flux_dir<3, false, UD>(acc, wz, vc, qsc, pc, p, q, C, 2);
         diss_apply(acc, t, C.dssp);
 #endif
     }
@@ -700,6 +700,9 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensor
 // Warps are decoupled: warp w owns row j0+w of the tile and never waits for
 // another warp except through the TMA ring (a slot is refilled by the last
 // warp to release it).
+// UD: the host verified dX1..dX5 are equal per axis (true for NAS), so one
+// d1 coefficient per axis suffices -- fewer uniform registers to reload.
+template <bool UD>
 __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensorMap *fmap,
                                          const Params &P) {
     // Extra CTAs beyond the compute grid (on SMs the lockstep schedule leaves
@@ -798,7 +801,7 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensor
         // One step body (instruction-cache footprint) and a register-move
         // rotation; unrolling by 5 for pure renaming measured slower (I$).
         for (int k = ka; k < kb; ++k) {
-            rhs_step<0>(g, P, umap, fmap, k);
+            rhs_step<0, UD>(g, P, umap, fmap, k);
 #pragma unroll
             for (int d = 0; d < 4; ++d) {
 #pragma unroll

@@ -70,10 +70,12 @@ struct Params {
 };
 
 // Launchers implemented in rhs_fast.cu / rhs_strict.cu.
+// uniform_d: every d1[ax][0..4] equal (NAS: dx1..dx5 = 0.75 ...), which lets
+// the kernel keep one d1 per axis in uniform registers.
 cudaError_t launch_rhs_fast(const CUtensorMap &umap, const CUtensorMap &fmap, const Params &p,
-                            cudaStream_t s);
+                            bool uniform_d, cudaStream_t s);
 cudaError_t launch_rhs_strict(const CUtensorMap &umap, const CUtensorMap &fmap, const Params &p,
-                              cudaStream_t s);
+                              bool uniform_d, cudaStream_t s);
 cudaError_t setup_rhs_fast(int *ctas_per_sm, cudaFuncAttributes *attr);
 cudaError_t setup_rhs_strict(int *ctas_per_sm, cudaFuncAttributes *attr);
 

@@ -90,6 +90,31 @@ def test_strict_bitwise_large(bench, cls):
     assert np.array_equal(g, o)
 
 
+@pytest.mark.parametrize("strict", [True, False])
+def test_general_coefficients(strict):
+    """Non-NAS coefficients (dX1..dX5 not all equal) take the general kernel
+    instead of the uniform-d1 specialisation; both sides get the same values."""
+    inp = nasgen.make_inputs(40, 27, 19, seed=8, B=1e-2, dt=0.002)
+    nz, ny, nx, _ = inp.u.shape
+    oc = oracle.set_constants(nx, ny, nz, inp.dt)
+    c = sr.coeffs_nas(nx, ny, nz, inp.dt)
+    for m, f in enumerate((1.0, 1.1, 0.9, 1.3, 0.7)):
+        setattr(oc, f"dx{m + 1}tx1", getattr(oc, f"dx{m + 1}tx1") * f)
+        setattr(oc, f"dz{m + 1}tz1", getattr(oc, f"dz{m + 1}tz1") * (2.0 - f))
+        c.dxt[m] = getattr(oc, f"dx{m + 1}tx1")
+        c.dzt[m] = getattr(oc, f"dz{m + 1}tz1")
+    o = oracle.compute_rhs(inp.u, inp.forcing, consts=oc)
+    du, df = sr.pack(inp.u), sr.pack(inp.forcing)
+    dr = torch.full_like(du, float("nan"))
+    sr.rhs(du, df, dr, nx, c, strict=strict)
+    torch.cuda.synchronize()
+    g = sr.unpack(dr, nx)
+    if strict:
+        assert np.array_equal(g, o)
+    else:
+        assert_tol(g, o)
+
+
 def test_exact_solution_residual_gpu():
     inp = nasgen.make_class("BT", "A", A=0.0)
     g = gpu_rhs(inp.u, inp.forcing, inp.dt, strict=False)
