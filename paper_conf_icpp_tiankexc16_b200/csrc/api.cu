@@ -13,9 +13,14 @@
 #include <cstdint>
 #include <cstdlib>
 #include <cstring>
+#include <cstdio>
 #include <mutex>
 
 #include "safara_internal.h"
+
+#ifndef SAFARA_TMA_SPLIT
+#define SAFARA_TMA_SPLIT 0
+#endif
 
 using namespace safara;
 
@@ -47,6 +52,8 @@ struct Tune {
     int l2promo = 0;
     int chunk = 0;
     int sched = 1;  // 0 = balanced contiguous ranges, 1 = lockstep (column, k-part)
+    int interleave = 1;  // lockstep CTA order: 1 = tile-major across CTAs, 0 = part-major
+    int face_ctas = 1;   // boundary faces on the idle SMs' extra CTAs (else by compute CTAs)
 } g_tune;
 
 int env_int(const char *name, int dflt) {
@@ -129,7 +136,7 @@ void to_coef(const safara_coeffs_t &in, Coef &c) {
 int encode_map(CUtensorMap *map, const double *base, const safara_dims_t &d, int nplanes,
                int box_x, int box_y, int *pos_j, int *pos_m, int *pos_k) {
     struct Ax { int which; long long stride, extent, box; } ax[3] = {
-        {0, d.sy, d.ny, box_y}, {1, d.sm, 5, 5}, {2, d.sk, nplanes, 1}};
+        {0, d.sy, d.ny, box_y}, {1, d.sm, 5, SAFARA_TMA_SPLIT ? 1 : 5}, {2, d.sk, nplanes, 1}};
     std::sort(ax, ax + 3, [](const Ax &a, const Ax &b) { return a.stride < b.stride; });
     cuuint64_t gdim[4] = {(cuuint64_t)d.nx, 0, 0, 0};
     cuuint64_t gstride[3];
@@ -202,6 +209,7 @@ int launch(const double *u, const double *f, double *r, const safara_dims_t &d, 
         // together, so neighbouring tiles read a plane's shared halo at the
         // same time and the second read hits L2.
         ncta = p.ncol * parts;
+        p.parts = g_tune.interleave ? (int)parts : 0;
     } else {
         ncta = (p.units + MIN_PLANES_PER_CTA - 1) / MIN_PLANES_PER_CTA;
         ncta = std::min(ncta, max_ctas);
@@ -212,9 +220,31 @@ int launch(const double *u, const double *f, double *r, const safara_dims_t &d, 
     }
     p.ncta = (int)ncta;
     // SMs the compute grid leaves idle take the boundary faces
-    p.nface_cta = (fk_hi > fk_lo && p.units > 0 && ncta < max_ctas)
+    p.nface_cta = (g_tune.face_ctas && fk_hi > fk_lo && p.units > 0 && ncta < max_ctas)
                       ? (int)std::min<long long>(max_ctas - ncta, 32) : 0;
 
+#ifdef SAFARA_TIMELINE
+    {   // debug builds only: a static per-CTA timestamp buffer, dumped at exit
+        static unsigned long long *buf = nullptr;
+        static int nct = 0;
+        if (!buf) {
+            cudaMalloc(&buf, 3 * 1024 * sizeof(unsigned long long));
+            std::atexit([] {
+                unsigned long long h[3 * 1024];
+                cudaDeviceSynchronize();
+                cudaMemcpy(h, buf, sizeof(h), cudaMemcpyDeviceToHost);
+                FILE *f = std::fopen("gpurun_out/timeline.txt", "w");
+                if (f) {
+                    for (int c = 0; c < nct; ++c)
+                        std::fprintf(f, "%d %llu %llu %llu\n", c, h[3 * c], h[3 * c + 1], h[3 * c + 2]);
+                    std::fclose(f);
+                }
+            });
+        }
+        p.dbg = buf;
+        nct = p.ncta + p.nface_cta;
+    }
+#endif
     CUtensorMap umap, fmap;
     int pj, pm, pk;
     rc = encode_map(&umap, u, d, nzu, UX, UY, &p.pos_j, &p.pos_m, &p.pos_k);
@@ -285,6 +315,8 @@ int safara_rhs_init(int device) {
     g_tune.l2promo = env_int("SAFARA_L2PROMO", g_tune.l2promo);
     g_tune.chunk = env_int("SAFARA_CHUNK", g_tune.chunk);
     g_tune.sched = env_int("SAFARA_SCHED", g_tune.sched);
+    g_tune.interleave = env_int("SAFARA_INTERLEAVE", g_tune.interleave);
+    g_tune.face_ctas = env_int("SAFARA_FACE_CTAS", g_tune.face_ctas);
     int major = 0, minor = 0, sms = 0;
     if (cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, device) ||
         cudaDeviceGetAttribute(&minor, cudaDevAttrComputeCapabilityMinor, device) ||

@@ -54,6 +54,15 @@
 #if SAFARA_ZETA_FIRST && SAFARA_PSUMS < 2
 #error "SAFARA_ZETA_FIRST reorders the accumulation: it needs SAFARA_PSUMS >= 2"
 #endif
+#ifndef SAFARA_TMA_SPLIT
+#define SAFARA_TMA_SPLIT 0  // 1: one TMA box per component (5 per field per plane)
+#endif
+#ifndef SAFARA_STORE_MODE
+#define SAFARA_STORE_MODE 0  // rhs stores: 0 st.global.cs, 1 default, 2 none (probe)
+#endif
+#ifndef SAFARA_PROBE
+#define SAFARA_PROBE 0  // 1: memory pipeline only, 2: compute only (roofline probes)
+#endif
 #ifndef SAFARA_L2PF
 #define SAFARA_L2PF 0  // planes beyond the ring to prefetch into L2 (0 = off)
 #endif
@@ -272,6 +281,24 @@ __device__ __forceinline__ void diss_terms(double (&t)[5], const double (&am2)[5
     }
 }
 
+// The five NAS cases along i as ONE instruction sequence: the coefficients of
+// a[i-1], a[i], a[i+1] come per lane from smem (-4/0, 6/5, -4/0) and an absent
+// a[i-2] / a[i+2] is read from a zero-filled (out-of-box) column.  fma(0,x,y)
+// = y, fma(-4,x,0) = -4x and c*a0 with c = 5 or 6 round exactly like the NAS
+// expressions, so the result is bit-identical to the generic select form.
+__device__ __forceinline__ void diss_terms_table(double (&t)[5], const double (&am2)[5],
+                                                 const double (&am1)[5], const double (&a0)[5],
+                                                 const double (&ap1)[5], const double (&ap2)[5],
+                                                 double cm1, double c0, double cp1) {
+#pragma unroll
+    for (int m = 0; m < 5; ++m) {
+        t[m] = __fma_rn(cm1, am1[m], am2[m]);
+        t[m] = t[m] + c0 * a0[m];
+        t[m] = __fma_rn(cp1, ap1[m], t[m]);
+        t[m] = t[m] + ap2[m];
+    }
+}
+
 __device__ __forceinline__ void diss_apply(double (&acc)[5], const double (&t)[5], double dssp) {
 #pragma unroll
     for (int m = 0; m < 5; ++m) acc[m] = acc[m] - dssp * t[m];
@@ -353,12 +380,26 @@ __device__ __forceinline__ void issue_plane(const CUtensorMap *umap, const CUten
     const int c3 = P.pos_j == 3 ? jc : (P.pos_m == 3 ? 0 : kb);
     double *dst = su + (size_t)slot * SLOT;
     mbar_expect_tx(&full[slot], with_f ? TMA_BYTES + TMA_BYTES_F : TMA_BYTES);
+#if SAFARA_TMA_SPLIT
+    // one box per component: more independent requests in flight per plane
+    for (int m = 0; m < 5; ++m) {
+        tma_load_4d(dst + m * UX * UY, umap, &full[slot], i0 - HX, P.pos_m == 1 ? m : c1,
+                    P.pos_m == 2 ? m : c2, P.pos_m == 3 ? m : c3);
+    }
+#else
     tma_load_4d(dst, umap, &full[slot], i0 - HX, c1, c2, c3);
+#endif
     if (with_f) {
         const int f1 = P.pos_j == 1 ? j0 : (P.pos_m == 1 ? 0 : kf);
         const int f2 = P.pos_j == 2 ? j0 : (P.pos_m == 2 ? 0 : kf);
         const int f3 = P.pos_j == 3 ? j0 : (P.pos_m == 3 ? 0 : kf);
+#if SAFARA_TMA_SPLIT
+        for (int m = 0; m < 5; ++m)
+            tma_load_4d(dst + U_SLOT + m * FX * TY, fmap, &full[slot], i0 - 1,
+                        P.pos_m == 1 ? m : f1, P.pos_m == 2 ? m : f2, P.pos_m == 3 ? m : f3);
+#else
         tma_load_4d(dst + U_SLOT, fmap, &full[slot], i0 - 1, f1, f2, f3);
+#endif
     }
 }
 
@@ -439,6 +480,12 @@ __device__ __forceinline__ uint64_t *smem_full() {
 __device__ __forceinline__ unsigned int *smem_released() {
     return reinterpret_cast<unsigned int *>(smem_full() + STAGES);
 }
+// Per-lane xi-dissipation coefficients of the current column tile:
+// [0][lane] = coefficient of a[i-1] (-4 or 0), [1][lane] = of a[i] (6 or 5),
+// [2][lane] = of a[i+1] (-4 or 0).
+__device__ __forceinline__ double *smem_xcoef() {
+    return reinterpret_cast<double *>(smem_ring() + (size_t)STAGES * SLOT + XCOEF_OFF);
+}
 
 struct Seg {
     double *rptr;  // rhs of (i, j, k, m=0) for the current step
@@ -475,10 +522,12 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensor
         for (int m = 0; m < 5; ++m) acc[m] = fs[(m * TY + g.ty) * FX + g.tx + 1];
     }
     // own column u(k+2) into the window; own rho_i / square of plane k+1
-    wait_plane(smem_full(), sq_k + 2);
+    if (SAFARA_PROBE != 2) wait_plane(smem_full(), sq_k + 2);
+#if SAFARA_PROBE != 3
     load5(g.w[PP], su + (size_t)((sq_k + 2) % STAGES) * SLOT, g.uc);
     if (g.in_grid) aux_of(g.w[PI][0], g.w[PI][1], g.w[PI][2], g.w[PI][3], g.ra[PI], g.sa[PI]);
     else { g.ra[PI] = 0.0; g.sa[PI] = 0.0; }
+#endif
     const double (&wz)[5] = g.w[Z];
     const double r0 = g.ra[Z], s0 = g.sa[Z];
     double vc[3];
@@ -487,6 +536,7 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensor
     vc[2] = wz[3] * r0;
     const double qsc = s0 * r0;
     const double pc = wz[4] * r0;
+#if SAFARA_PROBE != 1 && SAFARA_PROBE != 3
 #if SAFARA_ZETA_FIRST
     // zeta: everything from the register window (inter-iteration scalar
     // replacement along the sequential loop)
@@ -533,10 +583,19 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensor
         double t[5];
         {
             double pp[5], qq[5];
-            load5(pp, s, g.uc + 2);
-            load5(qq, s, g.uc - 2);
-            if (g.mid_x) diss_terms<false>(t, qq, q.u, wz, p.u, pp, Cases{});
-            else diss_terms<true>(t, qq, q.u, wz, p.u, pp, cases_of(g.i0 + g.tx, P.nx));
+            if (g.mid_x) {
+                load5(pp, s, g.uc + 2);
+                load5(qq, s, g.uc - 2);
+                diss_terms<false>(t, qq, q.u, wz, p.u, pp, Cases{});
+            } else {
+                // edge tile: absent i-2 / i+2 -> the zero-filled column beyond
+                const int i = g.i0 + g.tx;
+                load5(pp, s, g.uc + (i == P.nx - 3 ? 3 : 2));
+                load5(qq, s, g.uc - (i == 2 ? 3 : 2));
+                const double *xc = smem_xcoef();
+                diss_terms_table(t, qq, q.u, wz, p.u, pp, xc[g.tx], xc[TX + g.tx],
+                                 xc[2 * TX + g.tx]);
+            }
         }
         flux_dir<1, false, UD>(acc, wz, vc, qsc, pc, p, q, C, 0);
         diss_apply(acc, t, C.dssp);
@@ -596,10 +655,19 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensor
         double t[5];
         {
             double pp[5], qq[5];
-            load5(pp, s, g.uc + 2);
-            load5(qq, s, g.uc - 2);
-            if (g.mid_x) diss_terms<false>(t, qq, q.u, wz, p.u, pp, Cases{});
-            else diss_terms<true>(t, qq, q.u, wz, p.u, pp, cases_of(g.i0 + g.tx, P.nx));
+            if (g.mid_x) {
+                load5(pp, s, g.uc + 2);
+                load5(qq, s, g.uc - 2);
+                diss_terms<false>(t, qq, q.u, wz, p.u, pp, Cases{});
+            } else {
+                // edge tile: absent i-2 / i+2 -> the zero-filled column beyond
+                const int i = g.i0 + g.tx;
+                load5(pp, s, g.uc + (i == P.nx - 3 ? 3 : 2));
+                load5(qq, s, g.uc - (i == 2 ? 3 : 2));
+                const double *xc = smem_xcoef();
+                diss_terms_table(t, qq, q.u, wz, p.u, pp, xc[g.tx], xc[TX + g.tx],
+                                 xc[2 * TX + g.tx]);
+            }
         }
         flux_dir<1, false, UD>(acc, wz, vc, qsc, pc, p, q, C, 0);
         diss_apply(acc, t, C.dssp);
@@ -662,6 +730,15 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensor
 #endif
     }
 #endif
+#else
+#if SAFARA_PSUMS >= 2
+    for (int m = 0; m < 5; ++m) acc_z[m] = 0.0;
+#endif
+    {
+        __syncwarp();
+        if (g.tx == 0) { __threadfence_block(); rel_old = atomicAdd(&smem_released()[(int)(sq_k % STAGES)], 1u); }
+    }
+#endif
 #if SAFARA_PSUMS == 2
 #pragma unroll
     for (int m = 0; m < 5; ++m) acc[m] = acc[m] + acc_z[m];
@@ -669,19 +746,25 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensor
 #pragma unroll
     for (int m = 0; m < 5; ++m) acc[m] = acc[m] + (acc_y[m] + acc_z[m]);
 #endif
-    if (g.active) {
+    if (g.active && (SAFARA_PROBE != 2 || acc[0] == 1.2345e300)) {
         // rptr walks down the column one plane per step; the 5 component
         // planes are sm apart (one 64-bit pointer instead of 5 addresses)
         double *rp = g.rptr;
 #pragma unroll
         for (int m = 0; m < 5; ++m) {
+#if SAFARA_STORE_MODE == 0
             __stcs(rp, acc[m] * C.dt);
+#elif SAFARA_STORE_MODE == 1
+            *rp = acc[m] * C.dt;
+#elif SAFARA_STORE_MODE == 2
+            if (acc[m] == 1.2345e300) *rp = acc[m];  // probe: no stores
+#endif
             rp += P.sm;
         }
     }
     g.rptr += P.sk;
     // the last warp out of plane k (see the release above) refills its slot
-    if (g.tx == 0 && rel_old == (unsigned)(TY - 1)) {
+    if (SAFARA_PROBE != 2 && g.tx == 0 && rel_old == (unsigned)(TY - 1)) {
         smem_released()[(int)(sq_k % STAGES)] = 0;
         __threadfence_block();
         const int kn = k + STAGES;
@@ -705,10 +788,25 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensor
 template <bool UD>
 __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensorMap *fmap,
                                          const Params &P) {
+#ifdef SAFARA_TIMELINE
+    unsigned long long t_start;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_start));
+    unsigned smid;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+#endif
     // Extra CTAs beyond the compute grid (on SMs the lockstep schedule leaves
     // idle) only copy the boundary faces.
     if ((int)blockIdx.x >= P.ncta) {
         copy_faces(P, (int)blockIdx.x - P.ncta, P.nface_cta);
+#ifdef SAFARA_TIMELINE
+        if (threadIdx.x == 0 && P.dbg) {
+            unsigned long long t_end;
+            asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_end));
+            P.dbg[3 * blockIdx.x] = t_start;
+            P.dbg[3 * blockIdx.x + 1] = t_end;
+            P.dbg[3 * blockIdx.x + 2] = smid;
+        }
+#endif
         return;
     }
     double *su = smem_ring();
@@ -728,8 +826,17 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensor
     }
     __syncthreads();
 
-    int ub = split_point((int)blockIdx.x, P.units, P.ncta);
-    const int ue = split_point((int)blockIdx.x + 1, P.units, P.ncta);
+    int ub, ue;
+    if (P.parts > 0) {
+        // lockstep: CTA c owns column tile c % ncol, k-part c / ncol (all
+        // parts of one plane band run on CTAs spread over the whole chip)
+        const int c = (int)blockIdx.x, col = c % P.ncol, part = c / P.ncol;
+        ub = col * P.nplanes + (part * P.nplanes) / P.parts;
+        ue = col * P.nplanes + ((part + 1) * P.nplanes) / P.parts;
+    } else {
+        ub = split_point((int)blockIdx.x, P.units, P.ncta);
+        ue = split_point((int)blockIdx.x + 1, P.units, P.ncta);
+    }
 
 
     Seg g;
@@ -774,6 +881,14 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensor
 
         // Case flags (global indices, reading c12).
         g.mid_x = is_mid(g.i0, P.nx) && is_mid(g.i0 + TX - 1, P.nx);
+        if (!g.mid_x && tid < TX) {
+            const Cases cs = cases_of(g.i0 + tid, P.nx);
+            double *xc = smem_xcoef();
+            xc[tid] = cs.hm1 ? -4.0 : 0.0;
+            xc[TX + tid] = cs.five ? 5.0 : 6.0;
+            xc[2 * TX + tid] = cs.hp1 ? -4.0 : 0.0;
+        }
+        if (!g.mid_x) __syncthreads();  // the coefficient table is CTA-wide
         g.mid_y = is_mid(j, P.ny);
         g.uc = (g.ty + 2) * UX + (g.tx + HX);  // centre in the u tile
         g.ocol = i + P.sy * j;                  // own column offset (dim)
@@ -817,6 +932,15 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensor
         if (tid < STAGES) released[tid] = 0;
         __syncthreads();
     }
+#ifdef SAFARA_TIMELINE
+    if (tid == 0 && P.dbg) {
+        unsigned long long t_end;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_end));
+        P.dbg[3 * blockIdx.x] = t_start;
+        P.dbg[3 * blockIdx.x + 1] = t_end;
+        P.dbg[3 * blockIdx.x + 2] = smid;
+    }
+#endif
 }
 
 }  // namespace dev

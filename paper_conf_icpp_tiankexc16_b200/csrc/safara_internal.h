@@ -35,7 +35,9 @@ constexpr int F_PLANE = FX * TY * 5;
 constexpr int F_SLOT = ((F_PLANE * 8 + 127) / 128) * 128 / 8;
 constexpr uint32_t TMA_BYTES_F = F_PLANE * 8u;
 constexpr int SLOT = U_SLOT + F_SLOT;  // doubles per ring slot: u tile then forcing tile
-constexpr size_t SMEM_BYTES = (size_t)STAGES * SLOT * 8 + STAGES * 8 + STAGES * 4;
+constexpr int XCOEF_OFF = 16;  // doubles after the ring: mbarriers + counters first
+static_assert(STAGES * (8 + 4) <= XCOEF_OFF * 8, "mbarriers + release counters fit before the table");
+constexpr size_t SMEM_BYTES = (size_t)STAGES * SLOT * 8 + (XCOEF_OFF + 3 * TX) * 8;
 constexpr int MIN_PLANES_PER_CTA = 4;
 
 // Device-side coefficients: safara_coeffs_t plus the constant products that
@@ -60,12 +62,14 @@ struct Params {
     int chunk;             // planes per chunk of the chunk-major unit order
     int ncta;              // compute CTAs (the grid has ncta + nface_cta)
     int nface_cta;         // extra CTAs that only copy boundary faces (0: compute CTAs do it)
+    int parts;             // lockstep: k-parts per column (CTA c -> tile c % ncol); 0 = ranges
     int units;             // ncol*nplanes (column-plane work items, < 2^31)
     int fk_lo, fk_hi;      // local planes whose boundary faces this launch copies
     int pos_j, pos_m, pos_k;  // tensor-map dimension holding j, m, k
     const double *u;       // u buffer base (local plane 0)
     const double *f;       // forcing base (local plane 0)
     double *r;             // rhs base (local plane 0)
+    unsigned long long *dbg;  // SAFARA_TIMELINE builds: per-CTA {start, end, smid}
     Coef c;
 };
 
