@@ -178,6 +178,12 @@ int launch(const double *u, const double *f, double *r, const safara_dims_t &d, 
     std::memset(&p, 0, sizeof(p));
     p.nx = d.nx; p.ny = d.ny; p.nz = d.nz;
     p.sy = d.sy; p.sm = d.sm; p.sk = d.sk;
+    p.u_sy = p.f_sy = p.r_sy = d.sy;
+    p.u_sm = p.f_sm = p.r_sm = d.sm;
+    p.u_sk = p.f_sk = p.r_sk = d.sk;
+    p.u_sy64 = p.f_sy64 = p.r_sy64 = d.sy;
+    p.u_sm64 = p.f_sm64 = p.r_sm64 = d.sm;
+    p.u_sk64 = p.f_sk64 = p.r_sk64 = d.sk;
     p.k0 = k0; p.ukoff = ukoff; p.nzu = nzu;
     p.ka0 = ka0; p.kb0 = std::max(ka0, kb0);
     p.ka1 = ka1; p.kb1 = std::max(ka1, kb1);

@@ -71,6 +71,32 @@
 namespace safara {
 namespace dev {
 
+// ---- `dim` / `small` ablation (Table I/II replica) ----------
+// SAFARA_INDEX 0: one shared int32 descriptor for u/forcing/rhs (dim+small,
+// production); 1: a separate int32 descriptor per array (small only);
+// 2: separate int64 descriptors and 64-bit offsets per array (base).  The
+// host fills every copy with the same values, so results are identical.
+#ifndef SAFARA_INDEX
+#define SAFARA_INDEX 0
+#endif
+#if SAFARA_INDEX == 0
+typedef int idx_t;
+#define SY(a) P.sy
+#define SM(a) P.sm
+#define SK(a) P.sk
+#elif SAFARA_INDEX == 1
+typedef int idx_t;
+#define SY(a) P.a##_sy
+#define SM(a) P.a##_sm
+#define SK(a) P.a##_sk
+#else
+typedef long long idx_t;
+#define SY(a) (long long)P.a##_sy64
+#define SM(a) (long long)P.a##_sm64
+#define SK(a) (long long)P.a##_sk64
+#endif
+
+
 constexpr int UPM = UX * UY;  // doubles per component plane of a u tile
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) {
@@ -354,16 +380,16 @@ __device__ __forceinline__ void copy_faces(const Params &P, int cta, int nctas) 
                     i = 1 + r % (nx - 2);
                     j = 1 + r / (nx - 2);
                 }
-                off[b] = i + P.sy * j + P.sk * kl;
+                off[b] = i + SY(f) * j + SK(f) * kl;
 #pragma unroll
-                for (int m = 0; m < 5; ++m) v[b][m] = __ldcs(P.f + off[b] + P.sm * m);
+                for (int m = 0; m < 5; ++m) v[b][m] = __ldcs(P.f + off[b] + SM(f) * m);
             }
         }
 #pragma unroll
         for (int b = 0; b < FB; ++b)
             if (off[b] >= 0) {
 #pragma unroll
-                for (int m = 0; m < 5; ++m) __stcs(P.r + off[b] + P.sm * m, v[b][m]);
+                for (int m = 0; m < 5; ++m) __stcs(P.r + off[b] + SM(r) * m, v[b][m]);
             }
     }
 }
@@ -759,10 +785,10 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensor
 #elif SAFARA_STORE_MODE == 2
             if (acc[m] == 1.2345e300) *rp = acc[m];  // probe: no stores
 #endif
-            rp += P.sm;
+            rp += SM(r);
         }
     }
-    g.rptr += P.sk;
+    g.rptr += SK(r);
     // the last warp out of plane k (see the release above) refills its slot
     if (SAFARA_PROBE != 2 && g.tx == 0 && rel_old == (unsigned)(TY - 1)) {
         smem_released()[(int)(sq_k % STAGES)] = 0;
@@ -891,8 +917,8 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensor
         if (!g.mid_x) __syncthreads();  // the coefficient table is CTA-wide
         g.mid_y = is_mid(j, P.ny);
         g.uc = (g.ty + 2) * UX + (g.tx + HX);  // centre in the u tile
-        g.ocol = i + P.sy * j;                  // own column offset (dim)
-        g.rptr = P.r + (g.ocol + P.sk * (ka - P.k0));
+        g.ocol = i + SY(u) * j;                 // own column offset (dim)
+        g.rptr = P.r + ((idx_t)i + SY(r) * j + SK(r) * (ka - P.k0));
 
         // Window at rotation 0: planes ka-2, ka-1 from global memory (read
         // once per segment), ka and ka+1 from the TMA ring.
@@ -900,8 +926,8 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensor
             const int kbm2 = ka - 2 - P.k0 + P.ukoff, kbm1 = ka - 1 - P.k0 + P.ukoff;
 #pragma unroll
             for (int m = 0; m < 5; ++m) {
-                g.w[0][m] = (g.in_grid && kbm2 >= 0) ? __ldg(P.u + g.ocol + P.sm * m + P.sk * kbm2) : 0.0;
-                g.w[1][m] = (g.in_grid && kbm1 >= 0) ? __ldg(P.u + g.ocol + P.sm * m + P.sk * kbm1) : 0.0;
+                g.w[0][m] = (g.in_grid && kbm2 >= 0) ? __ldg(P.u + (idx_t)g.ocol + SM(u) * m + SK(u) * kbm2) : 0.0;
+                g.w[1][m] = (g.in_grid && kbm1 >= 0) ? __ldg(P.u + (idx_t)g.ocol + SM(u) * m + SK(u) * kbm1) : 0.0;
             }
             if (g.in_grid && kbm1 >= 0) aux_of(g.w[1][0], g.w[1][1], g.w[1][2], g.w[1][3], g.ra[1], g.sa[1]);
             else { g.ra[1] = 0.0; g.sa[1] = 0.0; }

@@ -52,6 +52,9 @@ struct Coef {
 struct Params {
     int nx, ny, nz;        // global extents
     int sy, sm, sk;        // shared element strides (dim clause), int32 (small)
+    // ablation copies (SAFARA_INDEX 1/2 builds only; same values)
+    int u_sy, u_sm, u_sk, f_sy, f_sm, f_sk, r_sy, r_sm, r_sk;
+    long long u_sy64, u_sm64, u_sk64, f_sy64, f_sm64, f_sk64, r_sy64, r_sm64, r_sk64;
     int k0;                // global k of forcing/rhs local plane 0
     int ukoff;             // u local plane = k - k0 + ukoff
     int nzu;               // planes in the u buffer
