@@ -11,60 +11,61 @@
 //    sequential k loop gets scalar replacement.
 //  * Inter-iteration scalar replacement along k, prioritised by reuse
 //    (cost model L x C): each u(m,i,j,k) is used at five
-//    consecutive k steps, so the thread keeps u(:,i,j,k-2..k+2) in a
-//    rotating register window (Fig. 6, generalised to depth 5),
-//    plus its own rho_i / square at k-1..k+1.  forcing is used once: it is
-//    streamed (one-step register prefetch), never staged.
+//    consecutive k steps.  The thread keeps u(:,i,j,k-1..k+1) plus its own
+//    rho_i / square of the same planes in a register window (Fig. 6,
+//    L895-914), and carries the zeta dissipation of plane k as the partial
+//    ((u[k-2] - 4u[k-1]) + 6u[k]), formed one step early in the NAS order, in
+//    place of a fifth plane.  The window rotates with period 3, so three
+//    unrolled steps rotate it by register renaming alone (no moves; the
+//    3-step body still fits the 32 KB instruction cache).
 //  * i/j neighbours (reused by 4 other threads each, the "uncoalesced"
 //    references SAFARA favours, L643-675) come from shared memory: the u
-//    plane tile with a halo of 2 arrives by TMA (cp.async.bulk.tensor, one
-//    box per plane, STAGES-deep mbarrier ring); rho_i and square of the
-//    plane (halo 1) are computed once per point into a 3-slot smem ring.
-//    Every other derived quantity (us, vs, ws, qs, u5*rho_i, products) is
-//    recomputed from {u, rho_i, square} at use: one DMUL costs a quarter of
-//    what a shared-memory double costs (64 FP64 lanes vs 16 doubles/clk/SM).
-//  * `dim`: forcing/rhs share one int32 descriptor (sy, sm, sk) held in the
+//    plane tile with a halo of 2 and the forcing tile arrive by TMA
+//    (cp.async.bulk.tensor, STAGES-deep mbarrier ring refilled by the last
+//    warp to release a slot).  rho_i / square of i+-1 come from the
+//    neighbour lanes (shuffles), of j+-1 are recomputed from the u values
+//    loaded for the stencil (rows belong to other warps; no cross-warp
+//    wait).  Every other derived quantity (us, vs, ws, qs, u5*rho_i,
+//    products) is recomputed at use from {u, rho_i, square}: one DMUL costs
+//    a quarter of a shared-memory double (64 FP64 lanes vs 16 doubles/clk/SM).
+//  * `dim`: u/forcing/rhs share one int32 descriptor (sy, sm, sk) held in the
 //    kernel parameters (constant bank); `small`: all offsets are 32-bit.
-//  * Evaluation order follows the NAS text left to right (DESIGN.md reading
-//    c6).  Where NAS multiplies by 2.0 or 4.0 (exact scalings) the subtract
-//    is a single fma, which rounds identically.
+//  * Evaluation order follows the NAS text left to right inside every
+//    stencil difference (reading c6).  Where NAS multiplies by 2.0
+//    or 4.0 (exact scalings) the subtract is a single fma, which rounds
+//    identically.
 #pragma once
 #include <cstdio>
+#include <type_traits>
 
 #include "safara_internal.h"
 
-// Production variant: number of independent partial sums the three
-// directions accumulate into (1 = the NAS chain; STRICT always uses 1).
-// Production only: form the zeta (register-only) partial sum first, while
-// the xi/eta shared-memory loads are in flight (needs PSUMS >= 2).  STRICT
-// keeps the NAS accumulation order forcing, xi, eta, zeta.
+// Production variant: the zeta (register-only) flux terms are accumulated
+// first, while the xi/eta shared-memory loads are in flight, and the zeta
+// dissipation last; STRICT keeps the NAS accumulation order forcing, xi,
+// eta, zeta (reading c6).  Both are one accumulation chain per
+// component.
 #if SAFARA_STRICT_BUILD
-#undef SAFARA_PSUMS
-#define SAFARA_PSUMS 1
-#undef SAFARA_ZETA_FIRST
 #define SAFARA_ZETA_FIRST 0
 #else
-#ifndef SAFARA_PSUMS
-#define SAFARA_PSUMS 2
-#endif
 #ifndef SAFARA_ZETA_FIRST
 #define SAFARA_ZETA_FIRST 1
 #endif
 #endif
-#if SAFARA_ZETA_FIRST && SAFARA_PSUMS < 2
-#error "SAFARA_ZETA_FIRST reorders the accumulation: it needs SAFARA_PSUMS >= 2"
-#endif
 #ifndef SAFARA_TMA_SPLIT
 #define SAFARA_TMA_SPLIT 0  // 1: one TMA box per component (5 per field per plane)
 #endif
-#ifndef SAFARA_STORE_MODE
-#define SAFARA_STORE_MODE 0  // rhs stores: 0 st.global.cs, 1 default, 2 none (probe)
-#endif
 #ifndef SAFARA_PROBE
-#define SAFARA_PROBE 0  // 1: memory pipeline only, 2: compute only (roofline probes)
+#define SAFARA_PROBE 0  // roofline probes: 1 memory only, 2 compute only (no TMA waits/refills, no stores), 3 no rhs stores
 #endif
-#ifndef SAFARA_L2PF
-#define SAFARA_L2PF 0  // planes beyond the ring to prefetch into L2 (0 = off)
+#ifndef SAFARA_STORE
+#define SAFARA_STORE 0  // rhs stores: 0 st.global.cs, 1 default caching, 2 none (probe)
+#endif
+// Production reciprocal: 0 = seed + 3 Newton steps (6 DFMA), 1 = seed + 2
+// Newton steps (4 DFMA), 2 = seed + one cubic step (3 DFMA; <= 1 ulp,
+// profiles/rcp_ulp_r01.txt).
+#ifndef SAFARA_RCP
+#define SAFARA_RCP 2
 #endif
 
 
@@ -166,21 +167,30 @@ __device__ __forceinline__ double d2(double ap, double ac, double aq) {
 }
 
 // Reciprocal.  STRICT: IEEE 1.0/x (correctly rounded, bit-identical to the
-// oracle).  Production: MUFU.RCP64H seed + three Newton steps, branch-free
-// (<= 1 ulp for the normal, positive densities of the path; the IEEE
-// division's special-case branch costs ~6 issue slots per call).
+// oracle).  Production: branch-free MUFU.RCP64H seed (about 20 good bits)
+// refined by FMA steps (the IEEE division's special-case branch costs ~6
+// issue slots per call; the densities of the path are normal and positive).
+// The cubic step r*(1 + e + e^2), e = 1 - x*r, takes the seed error to ~2^-60
+// before the final rounding (<= 1 ulp), in 3 DFMA instead of 2 Newton steps' 4.
 __device__ __forceinline__ double recip(double x) {
 #if SAFARA_STRICT_BUILD
     return 1.0 / x;
 #else
     double r;
     asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(r) : "d"(x));
+#if SAFARA_RCP == 2
+    const double e = __fma_rn(-x, r, 1.0);
+    return __fma_rn(r, __fma_rn(e, e, e), r);
+#else
     double e = __fma_rn(-x, r, 1.0);
     r = __fma_rn(r, e, r);
     e = __fma_rn(-x, r, 1.0);
+#if SAFARA_RCP == 0
     r = __fma_rn(r, e, r);
     e = __fma_rn(-x, r, 1.0);
+#endif
     return __fma_rn(r, e, r);
+#endif
 #endif
 }
 
@@ -276,7 +286,11 @@ __device__ __forceinline__ Cases cases_of(int x, int n) {
     return c;
 }
 
-__device__ __forceinline__ bool is_mid(int x, int n) { return x >= 3 && x <= n - 4; }
+// 3 <= x <= n-4 as one unsigned compare (n >= 6 is validated; n = 6 has no
+// mid points)
+__device__ __forceinline__ bool is_mid(int x, int n) {
+    return (unsigned)(x - 3) < (unsigned)(n - 6);
+}
 
 // The dissipation stencil value t_m (before `rhs -= dssp*t`).  It is formed
 // ahead of the flux terms (so the i+-2 / j+-2 neighbours die early: register
@@ -322,6 +336,34 @@ __device__ __forceinline__ void diss_terms_table(double (&t)[5], const double (&
         t[m] = t[m] + c0 * a0[m];
         t[m] = __fma_rn(cp1, ap1[m], t[m]);
         t[m] = t[m] + ap2[m];
+    }
+}
+
+// The five NAS cases along an axis whose case is warp-uniform (eta: one row
+// per warp), each written out as the NAS text evaluates it -- uniform
+// branches instead of per-element selects.  Case 0 is the interior form.
+__device__ __forceinline__ void diss_terms_case(double (&t)[5], const double (&am2)[5],
+                                                const double (&am1)[5], const double (&a0)[5],
+                                                const double (&ap1)[5], const double (&ap2)[5],
+                                                int c) {
+    if (c == 0) {
+#pragma unroll
+        for (int m = 0; m < 5; ++m)
+            t[m] = __fma_rn(-4.0, ap1[m], __fma_rn(-4.0, am1[m], am2[m]) + 6.0 * a0[m]) + ap2[m];
+    } else if (c == 1) {  // 5a[x] - 4a[x+1] + a[x+2]
+#pragma unroll
+        for (int m = 0; m < 5; ++m) t[m] = __fma_rn(-4.0, ap1[m], 5.0 * a0[m]) + ap2[m];
+    } else if (c == 2) {  // -4a[x-1] + 6a[x] - 4a[x+1] + a[x+2]
+#pragma unroll
+        for (int m = 0; m < 5; ++m)
+            t[m] = __fma_rn(-4.0, ap1[m], -4.0 * am1[m] + 6.0 * a0[m]) + ap2[m];
+    } else if (c == 3) {  // a[x-2] - 4a[x-1] + 6a[x] - 4a[x+1]
+#pragma unroll
+        for (int m = 0; m < 5; ++m)
+            t[m] = __fma_rn(-4.0, ap1[m], __fma_rn(-4.0, am1[m], am2[m]) + 6.0 * a0[m]);
+    } else {  // a[x-2] - 4a[x-1] + 5a[x]
+#pragma unroll
+        for (int m = 0; m < 5; ++m) t[m] = __fma_rn(-4.0, am1[m], am2[m]) + 5.0 * a0[m];
     }
 }
 
@@ -491,11 +533,13 @@ __device__ __forceinline__ void segment_of(const Params &P, int ub, int ue, int 
     }
 }
 
-// Per-segment state of one thread.  The register window is a 5-entry ring:
-// at rotation R, plane k-2+d lives in w[(R+d)%5] (d = 0..4) and its own
-// rho_i / square in ra/sa[(R+d)%5].  step<R> supports pure register renaming
-// (unroll by 5); the loop uses R = 0 plus explicit moves, which measured
-// faster because the 5x unrolled body overflows the instruction cache.
+// Per-segment state of one thread: the register window of the k march.
+// At rotation R (= step index mod 3) plane k-1 lives in a[R], plane k in
+// a[(R+1)%3] and plane k+1 in a[(R+2)%3]; plane k+2 is loaded into a[R] once
+// plane k-1 is dead, so three unrolled steps rotate the window by register
+// renaming alone (no moves).  The zeta dissipation of plane k is carried as
+// its partial ((a[k-2] - 4a[k-1]) + 6a[k]) -- formed one step early, in the
+// NAS order -- instead of keeping a fifth plane a[k-2].
 // Shared-memory carve-up (addresses are link-time constants, so nothing here
 // occupies a register across the loop).
 extern __shared__ __align__(128) unsigned char smem_raw[];
@@ -513,22 +557,53 @@ __device__ __forceinline__ double *smem_xcoef() {
     return reinterpret_cast<double *>(smem_ring() + (size_t)STAGES * SLOT + XCOEF_OFF);
 }
 
+// This CTA's unit range [ub, ue) and the current segment's end plane kb
+// live in shared memory across the k march (CTA-uniform; keeps registers free
+// for the unrolled window).
+__shared__ int s_range[7];  // ub, ue, segment kb, next segment's ub, tile i0, j0, segment ka
+__device__ __forceinline__ int smem_kb() { return *(volatile int *)&s_range[2]; }
+
 struct Seg {
     double *rptr;  // rhs of (i, j, k, m=0) for the current step
-    int i0, j0, ka, kb, uc, ocol, tx, ty;
-    bool in_grid, active, mid_x, mid_y;
-    uint32_t seq0;
-    double w[5][5];
-    double ra[5], sa[5];
+    int ka, kb;
+    int uc;         // own column's element offset in the u tile
+    int fo;         // own column's element offset in the forcing tile (= ty*FX + tx + 1)
+    bool lane0, lane31;
+    bool active, mid_x;
+    int ycase;      // NAS dissipation case of row j: 0 mid, 1 j=1, 2 j=2, 3 j=ny-3, 4 j=ny-2
+    uint32_t seq0;  // ring sequence number of the segment's first plane
+    double a[3][5];      // u(:, i, j, k-1..k+1), rotating (see above)
+    double ra[3], sa[3]; // rho_i / square of the same planes
+    double tp[5];        // zeta dissipation partial of plane k
 };
+
+// The zeta dissipation partial of plane kk: ((x2 - 4 x1) + c0 a0) with the
+// NAS case of kk selecting which neighbours exist (exact zero selection).
+__device__ __forceinline__ void zeta_partial(double (&tp)[5], const double (&am2)[5],
+                                             const double (&am1)[5], const double (&a0)[5],
+                                             int kk, int nz, bool mid) {
+    if (mid) {
+#pragma unroll
+        for (int m = 0; m < 5; ++m) tp[m] = __fma_rn(-4.0, am1[m], am2[m]) + 6.0 * a0[m];
+    } else {
+        const Cases c = cases_of(kk, nz);
+#pragma unroll
+        for (int m = 0; m < 5; ++m) {
+            const double x2 = c.hm2 ? am2[m] : 0.0;
+            const double x1 = c.hm1 ? am1[m] : 0.0;
+            const double cc = c.five ? 5.0 * a0[m] : 6.0 * a0[m];
+            tp[m] = __fma_rn(-4.0, x1, x2) + cc;
+        }
+    }
+}
 
 template <int R, bool UD>
 __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensorMap *umap,
                                          const CUtensorMap *fmap, int k) {
-    constexpr int QQ = R % 5, Q = (R + 1) % 5, Z = (R + 2) % 5, PI = (R + 3) % 5, PP = (R + 4) % 5;
+    constexpr int Q = R % 3, Z = (R + 1) % 3, PI = (R + 2) % 3;  // planes k-1, k, k+1
     const unsigned FULL = 0xffffffffu;
     const Coef &C = P.c;
-    const uint32_t sq_k = g.seq0 + (uint32_t)(k - g.ka);
+    const uint32_t sq_k = g.seq0 + (uint32_t)(k - g.ka);  // ring sequence number of plane k
     double *const su = smem_ring();
     const double *s = su + (size_t)(sq_k % STAGES) * SLOT;
 
@@ -536,25 +611,30 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensor
     // needs latency hiding, not a register slot)
     unsigned rel_old = 0;  // slot-release counter value seen by lane 0
     double acc[5];
-#if SAFARA_PSUMS >= 2
-    double acc_z[5];
-#endif
-#if SAFARA_PSUMS >= 3
-    double acc_y[5];
-#endif
     {
         const double *fs = s + U_SLOT;
 #pragma unroll
-        for (int m = 0; m < 5; ++m) acc[m] = fs[(m * TY + g.ty) * FX + g.tx + 1];
+        for (int m = 0; m < 5; ++m) acc[m] = fs[m * TY * FX + g.fo];
     }
-    // own column u(k+2) into the window; own rho_i / square of plane k+1
+    // plane k+2 must have landed: its own column enters the window at the
+    // end of this step (read from smem there, so it holds no registers
+    // across the step); own rho_i / square of plane k+1
     if (SAFARA_PROBE != 2) wait_plane(smem_full(), sq_k + 2);
-#if SAFARA_PROBE != 3
-    load5(g.w[PP], su + (size_t)((sq_k + 2) % STAGES) * SLOT, g.uc);
-    if (g.in_grid) aux_of(g.w[PI][0], g.w[PI][1], g.w[PI][2], g.w[PI][3], g.ra[PI], g.sa[PI]);
-    else { g.ra[PI] = 0.0; g.sa[PI] = 0.0; }
-#endif
-    const double (&wz)[5] = g.w[Z];
+    const double *const s2 = su + (size_t)((sq_k + 2) % STAGES) * SLOT;
+    aux_of(g.a[PI][0], g.a[PI][1], g.a[PI][2], g.a[PI][3], g.ra[PI], g.sa[PI]);
+
+    double an[5];
+#if SAFARA_PROBE == 1
+    load5(an, s2, g.uc);
+#pragma unroll
+    for (int m = 0; m < 5; ++m) acc[m] = acc[m] + an[m] * g.ra[PI] + s[g.uc + m * UPM];
+    __syncwarp();
+    if (g.lane0) {
+        __threadfence_block();
+        rel_old = atomicAdd(&smem_released()[(int)(sq_k % STAGES)], 1u);
+    }
+#else
+    const double (&wz)[5] = g.a[Z];
     const double r0 = g.ra[Z], s0 = g.sa[Z];
     double vc[3];
     vc[0] = wz[1] * r0;
@@ -562,32 +642,40 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensor
     vc[2] = wz[3] * r0;
     const double qsc = s0 * r0;
     const double pc = wz[4] * r0;
-#if SAFARA_PROBE != 1 && SAFARA_PROBE != 3
+
+    // zeta dissipation of plane k: the carried partial completed with
+    // u(k+1) and u(k+2) (uniform branch: edge planes only)
+    auto zeta_diss = [&](double (&t_z)[5]) {
+        if (is_mid(k, P.nz)) {
+#pragma unroll
+            for (int m = 0; m < 5; ++m) t_z[m] = __fma_rn(-4.0, g.a[PI][m], g.tp[m]) + an[m];
+        } else {
+            const Cases c = cases_of(k, P.nz);
+#pragma unroll
+            for (int m = 0; m < 5; ++m) {
+                const double y1 = c.hp1 ? g.a[PI][m] : 0.0;
+                const double y2 = c.hp2 ? an[m] : 0.0;
+                t_z[m] = __fma_rn(-4.0, y1, g.tp[m]) + y2;
+            }
+        }
+    };
+    auto zeta = [&]() {
+        Nb p, q;
+#pragma unroll
+        for (int m = 0; m < 5; ++m) {
+            p.u[m] = g.a[PI][m];
+            q.u[m] = g.a[Q][m];
+        }
+        p.rho = g.ra[PI]; p.sq = g.sa[PI];
+        q.rho = g.ra[Q]; q.sq = g.sa[Q];
+        flux_dir<3, false, UD>(acc, wz, vc, qsc, pc, p, q, C, 2);
+    };
 #if SAFARA_ZETA_FIRST
     // zeta: everything from the register window (inter-iteration scalar
-    // replacement along the sequential loop)
-    {
-        Nb p, q;
-#pragma unroll
-        for (int m = 0; m < 5; ++m) {
-            p.u[m] = g.w[PI][m];
-            q.u[m] = g.w[Q][m];
-        }
-        p.rho = g.ra[PI]; p.sq = g.sa[PI];
-        q.rho = g.ra[Q]; q.sq = g.sa[Q];
-        double t[5];
-        if (is_mid(k, P.nz))
-            diss_terms<false>(t, g.w[QQ], g.w[Q], wz, g.w[PI], g.w[PP], Cases{});
-        else
-            diss_terms<true>(t, g.w[QQ], g.w[Q], wz, g.w[PI], g.w[PP], cases_of(k, P.nz));
-#if SAFARA_PSUMS >= 2
-        flux_dir<3, true, UD>(acc_z, wz, vc, qsc, pc, p, q, C, 2);
-        diss_apply(acc_z, t, C.dssp);
-#else
-        flux_dir<3, false, UD>(acc, wz, vc, qsc, pc, p, q, C, 2);
-        diss_apply(acc, t, C.dssp);
+    // replacement along the sequential loop), while the xi/eta shared-memory
+    // loads are in flight
+    zeta();
 #endif
-    }
     // xi: rho_i/square of i+-1 are the neighbour lanes' own values; lanes 0
     // and 31 evaluate their outside neighbour themselves.
     {
@@ -599,12 +687,12 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensor
         q.rho = __shfl_up_sync(FULL, r0, 1);
         q.sq = __shfl_up_sync(FULL, s0, 1);
         {
-            const bool left = (g.tx == 0);
+            const bool left = g.lane0;
             double re, se;
             aux_of(left ? q.u[0] : p.u[0], left ? q.u[1] : p.u[1], left ? q.u[2] : p.u[2],
                    left ? q.u[3] : p.u[3], re, se);
             if (left) { q.rho = re; q.sq = se; }
-            if (g.tx == TX - 1) { p.rho = re; p.sq = se; }
+            if (g.lane31) { p.rho = re; p.sq = se; }
         }
         double t[5];
         {
@@ -615,25 +703,25 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensor
                 diss_terms<false>(t, qq, q.u, wz, p.u, pp, Cases{});
             } else {
                 // edge tile: absent i-2 / i+2 -> the zero-filled column beyond
-                const int i = g.i0 + g.tx;
-                load5(pp, s, g.uc + (i == P.nx - 3 ? 3 : 2));
-                load5(qq, s, g.uc - (i == 2 ? 3 : 2));
+                unsigned lane;  // = tx
+                asm("mov.u32 %0, %%laneid;" : "=r"(lane));
                 const double *xc = smem_xcoef();
-                diss_terms_table(t, qq, q.u, wz, p.u, pp, xc[g.tx], xc[TX + g.tx],
-                                 xc[2 * TX + g.tx]);
+                const int xo = reinterpret_cast<const int *>(xc + 3 * TX)[lane];
+                load5(pp, s, g.uc + (xo & 0xff));
+                load5(qq, s, g.uc - (xo >> 8));
+                diss_terms_table(t, qq, q.u, wz, p.u, pp, xc[lane], xc[TX + lane],
+                                 xc[2 * TX + lane]);
             }
         }
         flux_dir<1, false, UD>(acc, wz, vc, qsc, pc, p, q, C, 0);
         diss_apply(acc, t, C.dssp);
     }
     // eta: rows j+-1 belong to other warps; evaluate their rho_i / square
-    // from the u values loaded for the stencil.
+    // from the u values loaded for the stencil (no cross-warp dependency)
     {
         Nb p, q;
         load5(p.u, s, g.uc + UX);
         load5(q.u, s, g.uc - UX);
-        // rows j+-1 belong to other warps: evaluate their rho_i / square from
-        // the u values loaded for the stencil (no cross-warp dependency)
         aux_of(p.u[0], p.u[1], p.u[2], p.u[3], p.rho, p.sq);
         aux_of(q.u[0], q.u[1], q.u[2], q.u[3], q.rho, q.sq);
         double t[5];
@@ -641,167 +729,62 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensor
             double pp[5], qq[5];
             load5(pp, s, g.uc + 2 * UX);
             load5(qq, s, g.uc - 2 * UX);
-            if (g.mid_y) diss_terms<false>(t, qq, q.u, wz, p.u, pp, Cases{});
-            else diss_terms<true>(t, qq, q.u, wz, p.u, pp, cases_of(g.j0 + g.ty, P.ny));
+            diss_terms_case(t, qq, q.u, wz, p.u, pp, g.ycase);
         }
         // Every read of plane k's slot is done: release it now, act on the
         // counter at the end of the step (its latency hides behind eta).
         __syncwarp();
-        if (g.tx == 0) {
+        if (g.lane0) {
             __threadfence_block();
             rel_old = atomicAdd(&smem_released()[(int)(sq_k % STAGES)], 1u);
         }
-#if SAFARA_PSUMS >= 3
-        flux_dir<2, true, UD>(acc_y, wz, vc, qsc, pc, p, q, C, 1);
-        diss_apply(acc_y, t, C.dssp);
-#else
         flux_dir<2, false, UD>(acc, wz, vc, qsc, pc, p, q, C, 1);
         diss_apply(acc, t, C.dssp);
-#endif
     }
-#else
-    // xi: rho_i/square of i+-1 are the neighbour lanes' own values; lanes 0
-    // and 31 evaluate their outside neighbour themselves.
+#if !SAFARA_ZETA_FIRST
+    zeta();
+#endif
+    // u(k+2) completes the zeta dissipation of plane k (production applies
+    // it last, STRICT right after the zeta fluxes -- the NAS order)
+    load5(an, s2, g.uc);
     {
-        Nb p, q;
-        load5(p.u, s, g.uc + 1);
-        load5(q.u, s, g.uc - 1);
-        p.rho = __shfl_down_sync(FULL, r0, 1);
-        p.sq = __shfl_down_sync(FULL, s0, 1);
-        q.rho = __shfl_up_sync(FULL, r0, 1);
-        q.sq = __shfl_up_sync(FULL, s0, 1);
-        {
-            const bool left = (g.tx == 0);
-            double re, se;
-            aux_of(left ? q.u[0] : p.u[0], left ? q.u[1] : p.u[1], left ? q.u[2] : p.u[2],
-                   left ? q.u[3] : p.u[3], re, se);
-            if (left) { q.rho = re; q.sq = se; }
-            if (g.tx == TX - 1) { p.rho = re; p.sq = se; }
-        }
-        double t[5];
-        {
-            double pp[5], qq[5];
-            if (g.mid_x) {
-                load5(pp, s, g.uc + 2);
-                load5(qq, s, g.uc - 2);
-                diss_terms<false>(t, qq, q.u, wz, p.u, pp, Cases{});
-            } else {
-                // edge tile: absent i-2 / i+2 -> the zero-filled column beyond
-                const int i = g.i0 + g.tx;
-                load5(pp, s, g.uc + (i == P.nx - 3 ? 3 : 2));
-                load5(qq, s, g.uc - (i == 2 ? 3 : 2));
-                const double *xc = smem_xcoef();
-                diss_terms_table(t, qq, q.u, wz, p.u, pp, xc[g.tx], xc[TX + g.tx],
-                                 xc[2 * TX + g.tx]);
-            }
-        }
-        flux_dir<1, false, UD>(acc, wz, vc, qsc, pc, p, q, C, 0);
-        diss_apply(acc, t, C.dssp);
+        double t_z[5];
+        zeta_diss(t_z);
+        diss_apply(acc, t_z, C.dssp);
     }
-    // eta: rows j+-1 belong to other warps; evaluate their rho_i / square
-    // from the u values loaded for the stencil.
-    {
-        Nb p, q;
-        load5(p.u, s, g.uc + UX);
-        load5(q.u, s, g.uc - UX);
-        // rows j+-1 belong to other warps: evaluate their rho_i / square from
-        // the u values loaded for the stencil (no cross-warp dependency)
-        aux_of(p.u[0], p.u[1], p.u[2], p.u[3], p.rho, p.sq);
-        aux_of(q.u[0], q.u[1], q.u[2], q.u[3], q.rho, q.sq);
-        double t[5];
-        {
-            double pp[5], qq[5];
-            load5(pp, s, g.uc + 2 * UX);
-            load5(qq, s, g.uc - 2 * UX);
-            if (g.mid_y) diss_terms<false>(t, qq, q.u, wz, p.u, pp, Cases{});
-            else diss_terms<true>(t, qq, q.u, wz, p.u, pp, cases_of(g.j0 + g.ty, P.ny));
-        }
-        // Every read of plane k's slot is done: release it now, act on the
-        // counter at the end of the step (its latency hides behind eta).
-        __syncwarp();
-        if (g.tx == 0) {
-            __threadfence_block();
-            rel_old = atomicAdd(&smem_released()[(int)(sq_k % STAGES)], 1u);
-        }
-#if SAFARA_PSUMS >= 3
-        flux_dir<2, true, UD>(acc_y, wz, vc, qsc, pc, p, q, C, 1);
-        diss_apply(acc_y, t, C.dssp);
-#else
-        flux_dir<2, false, UD>(acc, wz, vc, qsc, pc, p, q, C, 1);
-        diss_apply(acc, t, C.dssp);
-#endif
-    }
-    // zeta: everything from the register window (inter-iteration scalar
-    // replacement along the sequential loop)
-    {
-        Nb p, q;
-#pragma unroll
-        for (int m = 0; m < 5; ++m) {
-            p.u[m] = g.w[PI][m];
-            q.u[m] = g.w[Q][m];
-        }
-        p.rho = g.ra[PI]; p.sq = g.sa[PI];
-        q.rho = g.ra[Q]; q.sq = g.sa[Q];
-        double t[5];
-        if (is_mid(k, P.nz))
-            diss_terms<false>(t, g.w[QQ], g.w[Q], wz, g.w[PI], g.w[PP], Cases{});
-        else
-            diss_terms<true>(t, g.w[QQ], g.w[Q], wz, g.w[PI], g.w[PP], cases_of(k, P.nz));
-#if SAFARA_PSUMS >= 2
-        flux_dir<3, true, UD>(acc_z, wz, vc, qsc, pc, p, q, C, 2);
-        diss_apply(acc_z, t, C.dssp);
-#else
-        flux_dir<3, false, UD>(acc, wz, vc, qsc, pc, p, q, C, 2);
-        diss_apply(acc, t, C.dssp);
-#endif
-    }
-#endif
-#else
-#if SAFARA_PSUMS >= 2
-    for (int m = 0; m < 5; ++m) acc_z[m] = 0.0;
-#endif
-    {
-        __syncwarp();
-        if (g.tx == 0) { __threadfence_block(); rel_old = atomicAdd(&smem_released()[(int)(sq_k % STAGES)], 1u); }
-    }
-#endif
-#if SAFARA_PSUMS == 2
-#pragma unroll
-    for (int m = 0; m < 5; ++m) acc[m] = acc[m] + acc_z[m];
-#elif SAFARA_PSUMS == 3
-#pragma unroll
-    for (int m = 0; m < 5; ++m) acc[m] = acc[m] + (acc_y[m] + acc_z[m]);
-#endif
-    if (g.active && (SAFARA_PROBE != 2 || acc[0] == 1.2345e300)) {
+#endif  // SAFARA_PROBE == 1
+    if (g.active && ((SAFARA_PROBE != 3 && SAFARA_PROBE != 2) || acc[0] == 1.2345e300)) {
         // rptr walks down the column one plane per step; the 5 component
         // planes are sm apart (one 64-bit pointer instead of 5 addresses)
         double *rp = g.rptr;
 #pragma unroll
         for (int m = 0; m < 5; ++m) {
-#if SAFARA_STORE_MODE == 0
+#if SAFARA_STORE == 0
             __stcs(rp, acc[m] * C.dt);
-#elif SAFARA_STORE_MODE == 1
+#elif SAFARA_STORE == 1
             *rp = acc[m] * C.dt;
-#elif SAFARA_STORE_MODE == 2
-            if (acc[m] == 1.2345e300) *rp = acc[m];  // probe: no stores
+#else
+            if (acc[m] == 1.2345e300) *rp = acc[m];
 #endif
             rp += SM(r);
         }
     }
     g.rptr += SK(r);
+    // the zeta partial of plane k+1 (plane k-1's last use), then rotate by
+    // renaming: plane k+2 takes the dead plane k-1's slot
+#if SAFARA_PROBE != 1
+    zeta_partial(g.tp, g.a[Q], g.a[Z], g.a[PI], k + 1, P.nz, is_mid(k + 1, P.nz));
+#endif
+#pragma unroll
+    for (int m = 0; m < 5; ++m) g.a[Q][m] = an[m];
     // the last warp out of plane k (see the release above) refills its slot
-    if (SAFARA_PROBE != 2 && g.tx == 0 && rel_old == (unsigned)(TY - 1)) {
+    if (SAFARA_PROBE != 2 && g.lane0 && rel_old == (unsigned)(TY - 1)) {
         smem_released()[(int)(sq_k % STAGES)] = 0;
         __threadfence_block();
-        const int kn = k + STAGES;
-        if (kn <= g.kb + 1)
-            issue_plane(umap, fmap, P, su, smem_full(), g.i0, g.j0, kn, kn < g.kb,
+        const int kn = k + STAGES, kb = smem_kb();  // segment end (read rarely)
+        if (kn <= kb + 1)
+            issue_plane(umap, fmap, P, su, smem_full(), s_range[4], s_range[5], kn, kn < kb,
                         sq_k + STAGES);
-#if SAFARA_L2PF > 0
-        if (kn + SAFARA_L2PF <= g.kb + 1)
-            prefetch_plane_l2(umap, fmap, P, g.i0, g.j0, kn + SAFARA_L2PF,
-                              kn + SAFARA_L2PF < g.kb);
-#endif
     }
 }
 
@@ -819,6 +802,7 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensor
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_start));
     unsigned smid;
     asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+    const long long c_start = clock64();
 #endif
     // Extra CTAs beyond the compute grid (on SMs the lockstep schedule leaves
     // idle) only copy the boundary faces.
@@ -830,7 +814,7 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensor
             asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_end));
             P.dbg[3 * blockIdx.x] = t_start;
             P.dbg[3 * blockIdx.x + 1] = t_end;
-            P.dbg[3 * blockIdx.x + 2] = smid;
+            P.dbg[3 * blockIdx.x + 2] = smid | ((unsigned long long)(clock64() - c_start) << 16);
         }
 #endif
         return;
@@ -864,10 +848,10 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensor
         ue = split_point((int)blockIdx.x + 1, P.units, P.ncta);
     }
 
-
     Seg g;
-    g.tx = tid % TX;
-    g.ty = tid / TX;  // lane = tx, warp = ty
+    g.lane0 = tid % TX == 0;
+    g.lane31 = tid % TX == TX - 1;
+    g.fo = (tid / TX) * FX + tid % TX + 1;
     g.seq0 = 0;
 
     // The first segment's planes are requested before the boundary-face copy
@@ -884,78 +868,104 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensor
     }
     if (P.nface_cta == 0) copy_faces(P, (int)blockIdx.x, P.ncta);
 
-    while (ub < ue) {
+    if (tid == 0) {
+        s_range[0] = ub;
+        s_range[1] = ue;
+    }
+    __syncthreads();
+    while (true) {
         // ---- segment: one column tile, a contiguous run of planes ----
+        ub = *(volatile int *)&s_range[0];
+        ue = *(volatile int *)&s_range[1];
+        if (ub >= ue) break;
         int col;
         segment_of(P, ub, ue, col, g.ka, g.kb);
-        ub += g.kb - g.ka;
+        // (re-read rather than kept live across the march)
+        unsigned tid_r;
+        asm volatile("mov.u32 %0, %%tid.x;" : "=r"(tid_r));
+        const int tx = (int)tid_r % TX, ty = (int)tid_r / TX;  // lane = tx, warp = ty
+        const int i0 = 1 + (col % P.ntx) * TX, j0 = 1 + (col / P.ntx) * TY;
+        if (tid == 0) {  // read by the refilling lane / at the segment end
+            s_range[2] = g.kb;
+            s_range[3] = ub + (g.kb - g.ka);
+            s_range[4] = i0;
+            s_range[5] = j0;
+            s_range[6] = g.ka;
+        }
         const int ka = g.ka, kb = g.kb;
 
-        g.i0 = 1 + (col % P.ntx) * TX;
-        g.j0 = 1 + (col / P.ntx) * TY;
-        const int i = g.i0 + g.tx, j = g.j0 + g.ty;
-        g.in_grid = (i < P.nx) && (j < P.ny);
+        const int i = i0 + tx, j = j0 + ty;
         g.active = (i <= P.nx - 2) && (j <= P.ny - 2);
-        const int nload = kb - ka + 2;  // planes ka .. kb+1
+        const int nload = kb - ka + 2;  // ring planes ka .. kb+1
 
         if (tid == 0 && !first) {
             const int npre = nload < STAGES ? nload : STAGES;
             for (int s = 0; s < npre; ++s)
-                issue_plane(umap, fmap, P, su, full, g.i0, g.j0, ka + s, ka + s < kb, g.seq0 + s);
+                issue_plane(umap, fmap, P, su, full, i0, j0, ka + s, ka + s < kb, g.seq0 + s);
         }
         first = false;
 
         // Case flags (global indices, reading c12).
-        g.mid_x = is_mid(g.i0, P.nx) && is_mid(g.i0 + TX - 1, P.nx);
+        g.mid_x = is_mid(i0, P.nx) && is_mid(i0 + TX - 1, P.nx);
         if (!g.mid_x && tid < TX) {
-            const Cases cs = cases_of(g.i0 + tid, P.nx);
+            const Cases cs = cases_of(i0 + tid, P.nx);
             double *xc = smem_xcoef();
             xc[tid] = cs.hm1 ? -4.0 : 0.0;
             xc[TX + tid] = cs.five ? 5.0 : 6.0;
             xc[2 * TX + tid] = cs.hp1 ? -4.0 : 0.0;
+            // offsets of a[i+2] / a[i-2], redirected to the zero-filled column
+            // beyond the box where NAS drops the term
+            reinterpret_cast<int *>(xc + 3 * TX)[tid] =
+                (i0 + tid == P.nx - 3 ? 3 : 2) | ((i0 + tid == 2 ? 3 : 2) << 8);
         }
         if (!g.mid_x) __syncthreads();  // the coefficient table is CTA-wide
-        g.mid_y = is_mid(j, P.ny);
-        g.uc = (g.ty + 2) * UX + (g.tx + HX);  // centre in the u tile
-        g.ocol = i + SY(u) * j;                 // own column offset (dim)
+        g.ycase = is_mid(j, P.ny) ? 0 : j == 1 ? 1 : j == 2 ? 2 : j == P.ny - 3 ? 3 : 4;
+        g.uc = (ty + 2) * UX + (tx + HX);  // centre in the u tile
         g.rptr = P.r + ((idx_t)i + SY(r) * j + SK(r) * (ka - P.k0));
 
-        // Window at rotation 0: planes ka-2, ka-1 from global memory (read
-        // once per segment), ka and ka+1 from the TMA ring.
+        // Window at rotation 0: planes ka-2 (only for the zeta partial) and
+        // ka-1 from global memory (read once per segment), ka and ka+1 from
+        // the TMA ring.  Lanes outside the grid read the nearest in-grid
+        // column (valid memory; they store nothing and feed no active lane).
         {
-            const int kbm2 = ka - 2 - P.k0 + P.ukoff, kbm1 = ka - 1 - P.k0 + P.ukoff;
+            const int ic = min(i, P.nx - 1), jc = min(j, P.ny - 1);
+            const int lk = ka - P.k0 + P.ukoff;  // local u plane of ka
+            const double *uc0 = P.u + (idx_t)(ic + SY(u) * jc);
 #pragma unroll
-            for (int m = 0; m < 5; ++m) {
-                g.w[0][m] = (g.in_grid && kbm2 >= 0) ? __ldg(P.u + (idx_t)g.ocol + SM(u) * m + SK(u) * kbm2) : 0.0;
-                g.w[1][m] = (g.in_grid && kbm1 >= 0) ? __ldg(P.u + (idx_t)g.ocol + SM(u) * m + SK(u) * kbm1) : 0.0;
+            for (int m = 0; m < 5; ++m)
+                g.a[0][m] = lk - 1 >= 0 ? __ldg(uc0 + SM(u) * m + SK(u) * (lk - 1)) : 0.0;
+            wait_plane(full, g.seq0);
+            load5(g.a[1], su + (size_t)(g.seq0 % STAGES) * SLOT, g.uc);
+            {
+                double am2[5];
+#pragma unroll
+                for (int m = 0; m < 5; ++m)
+                    am2[m] = lk - 2 >= 0 ? __ldg(uc0 + SM(u) * m + SK(u) * (lk - 2)) : 0.0;
+                zeta_partial(g.tp, am2, g.a[0], g.a[1], ka, P.nz, is_mid(ka, P.nz));
             }
-            if (g.in_grid && kbm1 >= 0) aux_of(g.w[1][0], g.w[1][1], g.w[1][2], g.w[1][3], g.ra[1], g.sa[1]);
-            else { g.ra[1] = 0.0; g.sa[1] = 0.0; }
+            aux_of(g.a[0][0], g.a[0][1], g.a[0][2], g.a[0][3], g.ra[0], g.sa[0]);
+            aux_of(g.a[1][0], g.a[1][1], g.a[1][2], g.a[1][3], g.ra[1], g.sa[1]);
+            wait_plane(full, g.seq0 + 1);
+            load5(g.a[2], su + (size_t)((g.seq0 + 1) % STAGES) * SLOT, g.uc);
         }
-        wait_plane(full, g.seq0);
-        load5(g.w[2], su + (size_t)(g.seq0 % STAGES) * SLOT, g.uc);
-        if (g.in_grid) aux_of(g.w[2][0], g.w[2][1], g.w[2][2], g.w[2][3], g.ra[2], g.sa[2]);
-        else { g.ra[2] = 0.0; g.sa[2] = 0.0; }
-        wait_plane(full, g.seq0 + 1);
-        load5(g.w[3], su + (size_t)((g.seq0 + 1) % STAGES) * SLOT, g.uc);
 
-        // One step body (instruction-cache footprint) and a register-move
-        // rotation; unrolling by 5 for pure renaming measured slower (I$).
-        for (int k = ka; k < kb; ++k) {
+        int k = ka;
+#pragma unroll 1
+        for (; k + 3 <= kb; k += 3) {
             rhs_step<0, UD>(g, P, umap, fmap, k);
-#pragma unroll
-            for (int d = 0; d < 4; ++d) {
-#pragma unroll
-                for (int m = 0; m < 5; ++m) g.w[d][m] = g.w[d + 1][m];
-                g.ra[d] = g.ra[d + 1];
-                g.sa[d] = g.sa[d + 1];
-            }
+            rhs_step<1, UD>(g, P, umap, fmap, k + 1);
+            rhs_step<2, UD>(g, P, umap, fmap, k + 2);
         }
-        g.seq0 += (uint32_t)nload;
+        if (k < kb) {
+            rhs_step<0, UD>(g, P, umap, fmap, k);
+            if (k + 1 < kb) rhs_step<1, UD>(g, P, umap, fmap, k + 1);
+        }
+        g.seq0 += (uint32_t)(s_range[2] - s_range[6] + 2);  // planes ka .. kb+1
         // Segment end: every warp has consumed every plane; planes kb, kb+1
         // were never released, so clear the counters before the next segment.
         __syncthreads();
         if (tid < STAGES) released[tid] = 0;
+        if (tid == 0) s_range[0] = s_range[3];
         __syncthreads();
     }
 #ifdef SAFARA_TIMELINE
@@ -964,7 +974,7 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensor
         asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_end));
         P.dbg[3 * blockIdx.x] = t_start;
         P.dbg[3 * blockIdx.x + 1] = t_end;
-        P.dbg[3 * blockIdx.x + 2] = smid;
+        P.dbg[3 * blockIdx.x + 2] = smid | ((unsigned long long)(clock64() - c_start) << 16);
     }
 #endif
 }

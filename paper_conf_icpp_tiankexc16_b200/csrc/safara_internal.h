@@ -37,7 +37,9 @@ constexpr uint32_t TMA_BYTES_F = F_PLANE * 8u;
 constexpr int SLOT = U_SLOT + F_SLOT;  // doubles per ring slot: u tile then forcing tile
 constexpr int XCOEF_OFF = 16;  // doubles after the ring: mbarriers + counters first
 static_assert(STAGES * (8 + 4) <= XCOEF_OFF * 8, "mbarriers + release counters fit before the table");
-constexpr size_t SMEM_BYTES = (size_t)STAGES * SLOT * 8 + (XCOEF_OFF + 3 * TX) * 8;
+// after the mbarriers: the edge-tile xi table, 3 coefficient rows (double)
+// and one row of packed i+-2 offsets (int)
+constexpr size_t SMEM_BYTES = (size_t)STAGES * SLOT * 8 + (XCOEF_OFF + 3 * TX + TX / 2) * 8;
 constexpr int MIN_PLANES_PER_CTA = 4;
 
 // Device-side coefficients: safara_coeffs_t plus the constant products that
