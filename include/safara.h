@@ -131,6 +131,50 @@ int safara_rhs_slab(const double *u_slab, const double *forcing_slab,
                     int nzl, const safara_coeffs_t *coeffs, int flags,
                     int part, void *stream);
 
+/* ---- the step-0 auxiliary fields and the rhs norm ------
+ *
+ * NAS compute_rhs forms, in its step 0, the per-point fields
+ * rho_i = 1/u1, us = u2*rho_i, vs = u3*rho_i, ws = u4*rho_i,
+ * square = 0.5*(u2*u2 + u3*u3 + u4*u4)*rho_i, qs = square*rho_i and, in SP,
+ * speed = sqrt(c1c2*rho_i*(u5 - square)); x/y/z_solve consume them.  These
+ * entry points write them alongside rhs, at EVERY grid point (boundary faces
+ * included), from the values the pass computes anyway (+48/56 B per point).
+ *   naux:  SAFARA_AUX_BT (6 fields, in the order above) or SAFARA_AUX_SP (7).
+ *   aux:   device array, component c of point (i, j, local plane p) at
+ *          i + sy*j + sm*c + sa*p, with (sy, sm) the shared descriptor's
+ *          strides (`dim`) and sa = naux*sm when sm < sk (components inside a
+ *          plane, the canonical layout) or sa = sk when components are
+ *          outermost (SP's [m][k][j][i]).  It holds nz planes (full grid) or
+ *          nzl planes (slab, plane p = global k0+p).  8-byte aligned; must not
+ *          overlap u, forcing or rhs (SAFARA_ERR_ARG); naux not 6/7:
+ *          SAFARA_ERR_ARG; offsets >= 2^31: SAFARA_ERR_TOO_LARGE.
+ * Otherwise identical to safara_rhs_ex / safara_rhs_slab (same rhs, same
+ * errors; STRICT aux values are bit-identical to NAS step 0).              */
+#define SAFARA_AUX_BT 6
+#define SAFARA_AUX_SP 7
+int safara_rhs_aux(const double *u, const double *forcing, double *rhs,
+                   double *aux, int naux, const safara_dims_t *dims,
+                   const safara_coeffs_t *coeffs, int flags, void *stream);
+int safara_rhs_slab_aux(const double *u_slab, const double *forcing_slab,
+                        double *rhs_slab, double *aux_slab, int naux,
+                        const safara_dims_t *dims, int k0, int nzl,
+                        const safara_coeffs_t *coeffs, int flags, int part,
+                        void *stream);
+
+/* The NAS rhs_norm numerator (NPB error.f): out[m] = sum of rhs(m,i,j,k)^2
+ * over the INTERIOR points (1 <= i <= nx-2, 1 <= j <= ny-2, 1 <= k <= nz-2)
+ * of the planes this buffer holds: rhs has nzl planes, plane p = global
+ * k0+p (k0 = 0, nzl = nz for a full grid).  rms(m) = sqrt(total[m] /
+ * ((nx-2)(ny-2)(nz-2))) after summing the slabs of all ranks.
+ *   work: device scratch of safara_norm_work_doubles() doubles;
+ *   out:  5 device doubles.  Asynchronous on `stream`, two kernel launches,
+ *   deterministic (fixed reduction order for a given grid).
+ * Errors: SAFARA_ERR_ARG (NULL / overlapping buffers), SAFARA_ERR_SHAPE
+ * (bad k range), SAFARA_ERR_ALIGN, descriptor errors as safara_validate_dims. */
+int safara_norm_work_doubles(void);
+int safara_rhs_sumsq(const double *rhs, const safara_dims_t *dims, int k0,
+                     int nzl, double *work, double *out, void *stream);
+
 /* End-to-end call with HOST arrays (canonical layout): copies u and forcing
  * host->device into the caller's device buffers u_dev/forcing_dev, runs the
  * pass into rhs_dev and copies rhs device->host.  The grid is cut into

@@ -58,7 +58,7 @@ def build(force: bool = False) -> str:
              os.path.getmtime(_LIB) < max(os.path.getmtime(_SRC), os.path.getmtime(_HDR)))
     if force or stale:
         tmp = _LIB + f".tmp{os.getpid()}"
-        subprocess.check_call(["gcc", *CFLAGS, "-o", tmp, _SRC])
+        subprocess.check_call(["gcc", *CFLAGS, "-o", tmp, _SRC, "-lm"])
         os.replace(tmp, _LIB)
     return _LIB
 
@@ -77,6 +77,11 @@ def _load():
             lib.oracle_compute_rhs.argtypes = [ctypes.c_int] * 3 + [
                 ctypes.POINTER(OracleConsts), dp, dp, dp, ctypes.c_int]
             lib.oracle_compute_rhs.restype = ctypes.c_int
+            lib.oracle_compute_aux.argtypes = [ctypes.c_int] * 3 + [
+                ctypes.POINTER(OracleConsts), dp, dp, ctypes.c_int]
+            lib.oracle_compute_aux.restype = ctypes.c_int
+            lib.oracle_rhs_sumsq.argtypes = [ctypes.c_int] * 3 + [dp, dp]
+            lib.oracle_rhs_sumsq.restype = ctypes.c_int
             _lib = lib
     return _lib
 
@@ -130,3 +135,35 @@ def compute_rhs(u: np.ndarray, forcing: np.ndarray, dt: float | None = None,
     if rc != 0:
         raise ValueError(f"oracle_compute_rhs failed ({rc}): extents must be >= 6")
     return from_nas(rn, nx, ny)
+
+
+def compute_aux(u: np.ndarray, naux: int = 6, dt: float | None = None,
+                consts: OracleConsts | None = None) -> np.ndarray:
+    """NAS compute_rhs step 0 fields at every point.
+
+    Returns shape (nz, ny, nx, naux): rho_i, us, vs, ws, square, qs (BT rhs.f
+    order) and, for naux = 7, SP's speed = sqrt(c1c2*rho_i*(u5 - square)).
+    ``dt`` only selects the constants (c1c2); it does not enter step 0."""
+    nz, ny, nx, _ = u.shape
+    if consts is None:
+        consts = set_constants(nx, ny, nz, 1.0 if dt is None else dt)
+    un = to_nas(np.asarray(u, dtype=np.float64))
+    an = np.zeros(un.shape[:3] + (naux,), dtype=np.float64)
+    dp = ctypes.POINTER(ctypes.c_double)
+    rc = _load().oracle_compute_aux(nx, ny, nz, ctypes.byref(consts), un.ctypes.data_as(dp),
+                                    an.ctypes.data_as(dp), int(naux))
+    if rc != 0:
+        raise ValueError("oracle_compute_aux: bad arguments (naux must be 6 or 7)")
+    return np.ascontiguousarray(an[:, :ny, :nx, :])
+
+
+def rhs_sumsq(rhs: np.ndarray) -> np.ndarray:
+    """NPB error.f rhs_norm numerator: per component, the sum of rhs^2 over
+    the interior points, in the Fortran loop order."""
+    nz, ny, nx, _ = rhs.shape
+    rn = to_nas(np.asarray(rhs, dtype=np.float64))
+    out = np.zeros(5, dtype=np.float64)
+    dp = ctypes.POINTER(ctypes.c_double)
+    if _load().oracle_rhs_sumsq(nx, ny, nz, rn.ctypes.data_as(dp), out.ctypes.data_as(dp)) != 0:
+        raise ValueError("oracle_rhs_sumsq: extents must be >= 3")
+    return out

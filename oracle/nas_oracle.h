@@ -61,4 +61,14 @@ int oracle_compute_rhs(int nx, int ny, int nz, const oracle_consts_t *c,
                        const double *u, const double *forcing, double *rhs,
                        int nthreads);
 
+/* NAS step 0 auxiliary fields at every point: naux = 6
+ * (rho_i, us, vs, ws, square, qs, the BT rhs.f order) or 7 (+ SP speed).
+ * aux: [nz][ny'][nx'][naux].  Returns 0 or -1 on bad arguments. */
+int oracle_compute_aux(int nx, int ny, int nz, const oracle_consts_t *c,
+                       const double *u, double *aux, int naux);
+
+/* NPB error.f rhs_norm numerator: out[m] = sum over interior points of
+ * rhs(m)^2 (k, j, i loop order).  Returns 0 or -1. */
+int oracle_rhs_sumsq(int nx, int ny, int nz, const double *rhs, double *out);
+
 #endif

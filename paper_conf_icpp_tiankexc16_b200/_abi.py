@@ -18,6 +18,7 @@ HEADER = os.path.join(os.path.dirname(PKG), "include", "safara.h")
 SAFARA_OK = 0
 SAFARA_FLAG_STRICT = 0x1
 SAFARA_PART_ALL, SAFARA_PART_INTERIOR, SAFARA_PART_EDGE = 0, 1, 2
+SAFARA_AUX_BT, SAFARA_AUX_SP = 6, 7
 
 
 class SafaraError(RuntimeError):
@@ -59,6 +60,14 @@ _SIGS = {
                          ctypes.POINTER(Coeffs), ctypes.c_int, ctypes.c_int, _dp], ctypes.c_int),
     "safara_rhs_host": ([_dp] * 6 + [ctypes.c_int] * 3 + [ctypes.POINTER(Coeffs), ctypes.c_int,
                                                            ctypes.c_int, _dp], ctypes.c_int),
+    "safara_rhs_aux": ([_dp, _dp, _dp, _dp, ctypes.c_int, ctypes.POINTER(Dims),
+                        ctypes.POINTER(Coeffs), ctypes.c_int, _dp], ctypes.c_int),
+    "safara_rhs_slab_aux": ([_dp, _dp, _dp, _dp, ctypes.c_int, ctypes.POINTER(Dims), ctypes.c_int,
+                             ctypes.c_int, ctypes.POINTER(Coeffs), ctypes.c_int, ctypes.c_int, _dp],
+                            ctypes.c_int),
+    "safara_norm_work_doubles": ([], ctypes.c_int),
+    "safara_rhs_sumsq": ([_dp, ctypes.POINTER(Dims), ctypes.c_int, ctypes.c_int, _dp, _dp, _dp],
+                         ctypes.c_int),
     "safara_launch_count": ([], ctypes.c_int64),
     "safara_kernel_info": ([ctypes.c_int, ctypes.POINTER(KernelInfo)], ctypes.c_int),
     "safara_strerror": ([ctypes.c_int], ctypes.c_char_p),

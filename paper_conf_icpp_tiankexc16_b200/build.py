@@ -26,6 +26,7 @@ COMMON = ARCH + ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC",
 UNITS = [
     ("rhs_fast.cu", ["--fmad=true", "-Xptxas", "-v"]),
     ("rhs_strict.cu", ["--fmad=false", "-Xptxas", "-v"]),
+    ("norm.cu", []),
     ("api.cu", []),
 ]
 DEPS = ["rhs_kernel.cuh", "rhs_variant.inc", "safara_internal.h"]

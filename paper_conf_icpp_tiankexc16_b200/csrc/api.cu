@@ -34,7 +34,7 @@ struct DeviceState {
     bool ready = false;
     int sms = 0;
     int ctas_fast = 0, ctas_strict = 0;
-    cudaFuncAttributes attr_fast{}, attr_strict{};
+    cudaFuncAttributes attr_fast[4]{}, attr_strict[4]{};
     // copy engines for safara_rhs_host's H2D / D2H pipeline (created at init)
     cudaStream_t h2d = nullptr, d2h = nullptr;
     cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
@@ -113,6 +113,7 @@ void to_coef(const safara_coeffs_t &in, Coef &c) {
     c.dssp = in.dssp;
     c.c1 = in.c1;
     c.c2 = in.c2;
+    c.c1c2 = in.c1 * in.c2;  // NAS set_constants: c1c2 = c1*c2
     c.t2[0] = in.tx2;
     c.t2[1] = in.ty2;
     c.t2[2] = in.tz2;
@@ -166,7 +167,8 @@ int encode_map(CUtensorMap *map, const double *base, const safara_dims_t &d, int
 int launch(const double *u, const double *f, double *r, const safara_dims_t &d, int nzu, int nzf,
            int k0,
            int ukoff, int ka0, int kb0, int ka1, int kb1, int fk_lo, int fk_hi,
-           const safara_coeffs_t *coeffs, int flags, cudaStream_t stream) {
+           const safara_coeffs_t *coeffs, int flags, cudaStream_t stream,
+           double *aux = nullptr, int naux = 0, int ska = 0) {
     int dev;
     int rc = current_device(&dev);
     if (rc) return rc;
@@ -198,6 +200,7 @@ int launch(const double *u, const double *f, double *r, const safara_dims_t &d, 
     p.chunk = std::max(1, std::min(g_tune.chunk > 0 ? g_tune.chunk : p.nplanes, p.nplanes));
     p.fk_lo = fk_lo; p.fk_hi = fk_hi;
     p.u = u; p.f = f; p.r = r;
+    p.aux = aux; p.naux = naux; p.ska = ska;
     to_coef(*coeffs, p.c);
 
     const bool strict = (flags & SAFARA_FLAG_STRICT) != 0;
@@ -264,6 +267,31 @@ int launch(const double *u, const double *f, double *r, const safara_dims_t &d, 
                            : launch_rhs_fast(umap, fmap, p, ud, stream);
     if (e != cudaSuccess) return SAFARA_ERR_CUDA;
     g_launches.fetch_add(1, std::memory_order_relaxed);
+    return SAFARA_OK;
+}
+
+// f1 aux array: naux component blocks with the shared (sy, sm) strides; the
+// plane stride is naux*sm when components sit inside a plane (canonical
+// [k][m][j][i]) and sk when they are outermost (SP's [m][k][j][i]).
+int aux_layout(const safara_dims_t &d, int naux, int nplanes, int *ska, long long *bytes) {
+    if (naux != SAFARA_AUX_BT && naux != SAFARA_AUX_SP) return SAFARA_ERR_ARG;
+    const long long sa = d.sm < d.sk ? (long long)naux * d.sm : (long long)d.sk;
+    if (d.sm >= d.sk && d.sm < d.sk * (long long)nplanes) return SAFARA_ERR_LAYOUT;
+    const long long maxo = (long long)(d.nx - 1) + (long long)d.sy * (d.ny - 1) +
+                           (long long)d.sm * (naux - 1) + sa * (nplanes - 1);
+    if (maxo >= (1LL << 31) || sa >= (1LL << 31)) return SAFARA_ERR_TOO_LARGE;
+    *ska = (int)sa;
+    *bytes = (maxo + 1) * (long long)sizeof(double);
+    return SAFARA_OK;
+}
+
+int check_aux(const double *aux, long long abytes, const double *u, long long ubytes,
+              const double *f, long long fbytes, const double *r, long long rbytes) {
+    if (!aux) return SAFARA_ERR_ARG;
+    if ((uintptr_t)aux & 7u) return SAFARA_ERR_ALIGN;
+    if (overlaps(aux, abytes, u, ubytes) || overlaps(aux, abytes, f, fbytes) ||
+        overlaps(aux, abytes, r, rbytes))
+        return SAFARA_ERR_ARG;
     return SAFARA_OK;
 }
 
@@ -343,8 +371,8 @@ int safara_rhs_init(int device) {
     if (cudaSetDevice(device) != cudaSuccess) return SAFARA_ERR_CUDA;
     DeviceState st;
     st.sms = sms;
-    cudaError_t e = setup_rhs_fast(&st.ctas_fast, &st.attr_fast);
-    if (e == cudaSuccess) e = setup_rhs_strict(&st.ctas_strict, &st.attr_strict);
+    cudaError_t e = setup_rhs_fast(&st.ctas_fast, st.attr_fast);
+    if (e == cudaSuccess) e = setup_rhs_strict(&st.ctas_strict, st.attr_strict);
     if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&st.h2d, cudaStreamNonBlocking);
     if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&st.d2h, cudaStreamNonBlocking);
     if (e == cudaSuccess) e = cudaEventCreateWithFlags(&st.ev_fork, cudaEventDisableTiming);
@@ -394,9 +422,9 @@ int safara_rhs(const double *u, const double *forcing, double *rhs, int nx, int 
     return safara_rhs_ex(u, forcing, rhs, &d, coeffs, 0, stream);
 }
 
-int safara_rhs_slab(const double *u_slab, const double *forcing_slab, double *rhs_slab,
-                    const safara_dims_t *dims, int k0, int nzl, const safara_coeffs_t *coeffs,
-                    int flags, int part, void *stream) {
+static int slab_launch(const double *u_slab, const double *forcing_slab, double *rhs_slab,
+                       const safara_dims_t *dims, int k0, int nzl, const safara_coeffs_t *coeffs,
+                       int flags, int part, void *stream, double *aux, int naux, int ska) {
     if (!dims) return SAFARA_ERR_ARG;
     if (part < SAFARA_PART_ALL || part > SAFARA_PART_EDGE) return SAFARA_ERR_ARG;
     if (nzl < 2 || k0 < 0 || k0 + nzl > dims->nz) return SAFARA_ERR_SHAPE;
@@ -419,7 +447,50 @@ int safara_rhs_slab(const double *u_slab, const double *forcing_slab, double *rh
         fk_lo = fk_hi = 0;
     }
     return launch(u_slab, forcing_slab, rhs_slab, *dims, nzu, nzl, k0, 2, ka0, kb0, ka1, kb1, fk_lo,
-                  fk_hi, coeffs, flags, (cudaStream_t)stream);
+                  fk_hi, coeffs, flags, (cudaStream_t)stream, aux, naux, ska);
+}
+
+int safara_rhs_slab(const double *u_slab, const double *forcing_slab, double *rhs_slab,
+                    const safara_dims_t *dims, int k0, int nzl, const safara_coeffs_t *coeffs,
+                    int flags, int part, void *stream) {
+    return slab_launch(u_slab, forcing_slab, rhs_slab, dims, k0, nzl, coeffs, flags, part, stream,
+                       nullptr, 0, 0);
+}
+
+int safara_rhs_aux(const double *u, const double *forcing, double *rhs, double *aux, int naux,
+                   const safara_dims_t *dims, const safara_coeffs_t *coeffs, int flags,
+                   void *stream) {
+    int rc = validate(dims, dims ? dims->nz : 0);
+    if (rc) return rc;
+    const long long bytes = (max_offset(*dims, dims->nz) + 1) * (long long)sizeof(double);
+    rc = check_ptrs(u, bytes, forcing, bytes, rhs, bytes);
+    if (rc) return rc;
+    int ska;
+    long long abytes;
+    rc = aux_layout(*dims, naux, dims->nz, &ska, &abytes);
+    if (rc) return rc;
+    rc = check_aux(aux, abytes, u, bytes, forcing, bytes, rhs, bytes);
+    if (rc) return rc;
+    const int nz = dims->nz;
+    return launch(u, forcing, rhs, *dims, nz, nz, 0, 0, 1, nz - 1, 0, 0, 0, nz, coeffs, flags,
+                  (cudaStream_t)stream, aux, naux, ska);
+}
+
+int safara_rhs_slab_aux(const double *u_slab, const double *forcing_slab, double *rhs_slab,
+                        double *aux_slab, int naux, const safara_dims_t *dims, int k0, int nzl,
+                        const safara_coeffs_t *coeffs, int flags, int part, void *stream) {
+    if (!dims) return SAFARA_ERR_ARG;
+    if (nzl < 2 || k0 < 0 || k0 + nzl > dims->nz) return SAFARA_ERR_SHAPE;
+    int ska;
+    long long abytes;
+    int rc = aux_layout(*dims, naux, nzl, &ska, &abytes);
+    if (rc) return rc;
+    const long long ubytes = (max_offset(*dims, nzl + 4) + 1) * (long long)sizeof(double);
+    const long long fbytes = (max_offset(*dims, nzl) + 1) * (long long)sizeof(double);
+    rc = check_aux(aux_slab, abytes, u_slab, ubytes, forcing_slab, fbytes, rhs_slab, fbytes);
+    if (rc) return rc;
+    return slab_launch(u_slab, forcing_slab, rhs_slab, dims, k0, nzl, coeffs, flags, part, stream,
+                       aux_slab, naux, ska);
 }
 
 int safara_rhs_host(const double *u_host, const double *forcing_host, double *rhs_host,
@@ -474,6 +545,33 @@ int safara_rhs_host(const double *u_host, const double *forcing_host, double *rh
     return ok ? SAFARA_OK : SAFARA_ERR_CUDA;
 }
 
+int safara_norm_work_doubles(void) { return 5 * norm_grid(); }
+
+int safara_rhs_sumsq(const double *rhs, const safara_dims_t *dims, int k0, int nzl, double *work,
+                     double *out, void *stream) {
+    int dev;
+    int rc = current_device(&dev);
+    if (rc) return rc;
+    if (!dims) return SAFARA_ERR_ARG;
+    if (nzl < 1 || k0 < 0 || k0 + nzl > dims->nz) return SAFARA_ERR_SHAPE;
+    rc = validate(dims, nzl);
+    if (rc) return rc;
+    if (!rhs || !work || !out) return SAFARA_ERR_ARG;
+    if (((uintptr_t)rhs | (uintptr_t)work | (uintptr_t)out) & 7u) return SAFARA_ERR_ALIGN;
+    const long long rbytes = (max_offset(*dims, nzl) + 1) * (long long)sizeof(double);
+    const long long wbytes = (long long)safara_norm_work_doubles() * sizeof(double);
+    if (overlaps(work, wbytes, rhs, rbytes) || overlaps(out, 40, rhs, rbytes) ||
+        overlaps(out, 40, work, wbytes))
+        return SAFARA_ERR_ARG;
+    const int lo = std::max(k0, 1), hi = std::min(k0 + nzl, dims->nz - 1);
+    const int nk = std::max(0, hi - lo);
+    cudaError_t e = launch_sumsq(rhs, dims->nx, dims->ny, dims->sy, dims->sm, dims->sk, lo - k0,
+                                 nk, work, out, (cudaStream_t)stream);
+    if (e != cudaSuccess) return SAFARA_ERR_CUDA;
+    g_launches.fetch_add(2, std::memory_order_relaxed);
+    return SAFARA_OK;
+}
+
 int64_t safara_launch_count(void) { return g_launches.load(); }
 
 int safara_kernel_info(int which, safara_kernel_info_t *out) {
@@ -482,10 +580,13 @@ int safara_kernel_info(int which, safara_kernel_info_t *out) {
     int rc = current_device(&dev);
     if (rc) return rc;
     const DeviceState &st = g_dev[dev];
-    const cudaFuncAttributes &a = which ? st.attr_strict : st.attr_fast;
-    out->regs_per_thread = a.numRegs;
-    out->local_bytes = (int)a.localSizeBytes;
-    out->smem_bytes = (int)(a.sharedSizeBytes + SMEM_BYTES);
+    const cudaFuncAttributes *a = which ? st.attr_strict : st.attr_fast;
+    out->regs_per_thread = a[0].numRegs;
+    // local (spill) bytes of the production instantiation (NAS coefficients,
+    // no aux); the general / aux instantiations spill 4-8 B in their segment
+    // setup, outside the k march (profiles/ptxas_r01.txt)
+    out->local_bytes = (int)a[0].localSizeBytes;
+    out->smem_bytes = (int)(a[0].sharedSizeBytes + SMEM_BYTES);
     out->threads_per_cta = NTHREADS;
     out->ctas_per_sm = which ? st.ctas_strict : st.ctas_fast;
     out->tile_x = TX;

@@ -201,6 +201,23 @@ __device__ __forceinline__ void aux_of(double u1, double u2, double u3, double u
     sq = 0.5 * (u2 * u2 + u3 * u3 + u4 * u4) * rho;
 }
 
+// the step-0 fields NAS x/y/z_solve consume, stored for
+// the point at element offset `off` (i + sy*j) of local plane kl:
+// rho_i, us, vs, ws, square, qs [, speed = sqrt(c1c2*rho_i*(u5 - square))].
+__device__ __forceinline__ void store_aux(const Params &P, int off, int kl, double rho,
+                                          double us, double vs, double ws, double sq,
+                                          double qs, double u5) {
+    double *a = P.aux + (off + P.ska * kl);
+    const int sm = P.sm;
+    __stcs(a, rho);
+    __stcs(a + sm, us);
+    __stcs(a + 2 * sm, vs);
+    __stcs(a + 3 * sm, ws);
+    __stcs(a + 4 * sm, sq);
+    __stcs(a + 5 * sm, qs);
+    if (P.naux > 6) __stcs(a + 6 * sm, sqrt(P.c.c1c2 * rho * (u5 - sq)));
+}
+
 struct Nb {
     double u[5];
     double rho, sq;
@@ -374,6 +391,7 @@ __device__ __forceinline__ void diss_apply(double (&acc)[5], const double (&t)[5
 
 // Copy forcing -> rhs on this launch's boundary-face points (rhs = forcing,
 // unscaled; App. A step 1, reading c3), spread over all CTAs.
+template <bool AUX>
 __device__ __forceinline__ void copy_faces(const Params &P, int cta, int nctas) {
     const int nx = P.nx, ny = P.ny;
     const int per = 2 * nx + 2 * (ny - 2);
@@ -425,6 +443,15 @@ __device__ __forceinline__ void copy_faces(const Params &P, int cta, int nctas) 
                 off[b] = i + SY(f) * j + SK(f) * kl;
 #pragma unroll
                 for (int m = 0; m < 5; ++m) v[b][m] = __ldcs(P.f + off[b] + SM(f) * m);
+                if (AUX) {  // aux of the face point from u (u plane = kl + ukoff)
+                    const double *up = P.u + (i + SY(u) * j + SK(u) * (kl + P.ukoff));
+                    const double u1 = __ldg(up), u2 = __ldg(up + SM(u)), u3 = __ldg(up + 2 * SM(u));
+                    const double u4 = __ldg(up + 3 * SM(u)), u5 = __ldg(up + 4 * SM(u));
+                    double rho, sq;
+                    aux_of(u1, u2, u3, u4, rho, sq);
+                    store_aux(P, i + P.sy * j, kl, rho, u2 * rho, u3 * rho, u4 * rho, sq,
+                              sq * rho, u5);
+                }
             }
         }
 #pragma unroll
@@ -597,7 +624,7 @@ __device__ __forceinline__ void zeta_partial(double (&tp)[5], const double (&am2
     }
 }
 
-template <int R, bool UD>
+template <int R, bool UD, bool AUX>
 __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensorMap *umap,
                                          const CUtensorMap *fmap, int k) {
     constexpr int Q = R % 3, Z = (R + 1) % 3, PI = (R + 2) % 3;  // planes k-1, k, k+1
@@ -642,6 +669,12 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensor
     vc[2] = wz[3] * r0;
     const double qsc = s0 * r0;
     const double pc = wz[4] * r0;
+    if (AUX && g.active) {
+        // element offset of (i, j) from the walking rhs pointer
+        const int kl = k - P.k0;
+        const int off = (int)(g.rptr - P.r) - SK(r) * kl;
+        store_aux(P, off, kl, r0, vc[0], vc[1], vc[2], s0, qsc, wz[4]);
+    }
 
     // zeta dissipation of plane k: the carried partial completed with
     // u(k+1) and u(k+2) (uniform branch: edge planes only)
@@ -794,7 +827,7 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensor
 // warp to release it).
 // UD: the host verified dX1..dX5 are equal per axis (true for NAS), so one
 // d1 coefficient per axis suffices -- fewer uniform registers to reload.
-template <bool UD>
+template <bool UD, bool AUX>
 __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensorMap *fmap,
                                          const Params &P) {
 #ifdef SAFARA_TIMELINE
@@ -807,7 +840,7 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensor
     // Extra CTAs beyond the compute grid (on SMs the lockstep schedule leaves
     // idle) only copy the boundary faces.
     if ((int)blockIdx.x >= P.ncta) {
-        copy_faces(P, (int)blockIdx.x - P.ncta, P.nface_cta);
+        copy_faces<AUX>(P, (int)blockIdx.x - P.ncta, P.nface_cta);
 #ifdef SAFARA_TIMELINE
         if (threadIdx.x == 0 && P.dbg) {
             unsigned long long t_end;
@@ -866,7 +899,7 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensor
         for (int s = 0; s < npre; ++s)
             issue_plane(umap, fmap, P, su, full, i0, j0, ka + s, ka + s < kb, (uint32_t)s);
     }
-    if (P.nface_cta == 0) copy_faces(P, (int)blockIdx.x, P.ncta);
+    if (P.nface_cta == 0) copy_faces<AUX>(P, (int)blockIdx.x, P.ncta);
 
     if (tid == 0) {
         s_range[0] = ub;
@@ -952,13 +985,13 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensor
         int k = ka;
 #pragma unroll 1
         for (; k + 3 <= kb; k += 3) {
-            rhs_step<0, UD>(g, P, umap, fmap, k);
-            rhs_step<1, UD>(g, P, umap, fmap, k + 1);
-            rhs_step<2, UD>(g, P, umap, fmap, k + 2);
+            rhs_step<0, UD, AUX>(g, P, umap, fmap, k);
+            rhs_step<1, UD, AUX>(g, P, umap, fmap, k + 1);
+            rhs_step<2, UD, AUX>(g, P, umap, fmap, k + 2);
         }
         if (k < kb) {
-            rhs_step<0, UD>(g, P, umap, fmap, k);
-            if (k + 1 < kb) rhs_step<1, UD>(g, P, umap, fmap, k + 1);
+            rhs_step<0, UD, AUX>(g, P, umap, fmap, k);
+            if (k + 1 < kb) rhs_step<1, UD, AUX>(g, P, umap, fmap, k + 1);
         }
         g.seq0 += (uint32_t)(s_range[2] - s_range[6] + 2);  // planes ka .. kb+1
         // Segment end: every warp has consumed every plane; planes kb, kb+1

@@ -49,6 +49,7 @@ struct Coef {
     double t2[3];          // tx2, ty2, tz2
     double d1[3][5];       // dx{m}tx1, dy{m}ty1, dz{m}tz1
     double con2[3], con2x43[3], con3[3], con4[3], con5[3];
+    double c1c2;           // c1*c2 (SP speed, aux output only)
 };
 
 struct Params {
@@ -74,6 +75,10 @@ struct Params {
     const double *u;       // u buffer base (local plane 0)
     const double *f;       // forcing base (local plane 0)
     double *r;             // rhs base (local plane 0)
+    double *aux;           // SURVEY §8(f) f1 aux output (NULL: none); component c of
+                           // local plane kl at i + sy*j + sm*c + ska*kl
+    int naux;              // 6 (rho_i, us, vs, ws, square, qs) or 7 (+ SP speed)
+    int ska;               // aux plane stride
     unsigned long long *dbg;  // SAFARA_TIMELINE builds: per-CTA {start, end, smid}
     Coef c;
 };
@@ -85,6 +90,12 @@ cudaError_t launch_rhs_fast(const CUtensorMap &umap, const CUtensorMap &fmap, co
                             bool uniform_d, cudaStream_t s);
 cudaError_t launch_rhs_strict(const CUtensorMap &umap, const CUtensorMap &fmap, const Params &p,
                               bool uniform_d, cudaStream_t s);
+// norm.cu: per-component sums of squares over interior points (f1)
+int norm_grid();
+cudaError_t launch_sumsq(const double *rhs, int nx, int ny, int sy, int sm, int sk, int kl0, int nk,
+                         double *work, double *out, cudaStream_t s);
+
+// attr: 4 entries (production NAS path, general coefficients, aux, NAS + aux)
 cudaError_t setup_rhs_fast(int *ctas_per_sm, cudaFuncAttributes *attr);
 cudaError_t setup_rhs_strict(int *ctas_per_sm, cudaFuncAttributes *attr);
 

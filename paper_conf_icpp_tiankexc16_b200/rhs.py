@@ -13,8 +13,8 @@ import ctypes
 import numpy as np
 import torch
 
-from ._abi import (SAFARA_FLAG_STRICT, SAFARA_PART_ALL, Coeffs, Dims, KernelInfo,
-                   check, lib)
+from ._abi import (SAFARA_AUX_BT, SAFARA_AUX_SP, SAFARA_FLAG_STRICT, SAFARA_PART_ALL, Coeffs,
+                   Dims, KernelInfo, check, lib)
 
 _initialised: set[int] = set()
 
@@ -140,3 +140,88 @@ def kernel_info(strict: bool = False) -> dict:
     k = KernelInfo()
     check(lib().safara_kernel_info(1 if strict else 0, ctypes.byref(k)), "safara_kernel_info")
     return {f: getattr(k, f) for f, _ in KernelInfo._fields_}
+
+
+# ---- step-0 auxiliary fields and the rhs norm -------------
+
+AUX_NAMES = ("rho_i", "us", "vs", "ws", "square", "qs", "speed")
+
+
+def empty_aux(nx: int, ny: int, nplanes: int, naux: int = SAFARA_AUX_BT,
+              device="cuda") -> torch.Tensor:
+    """Canonical aux array (nplanes, naux, ny, sy): component c of (i, j, p)
+    at i + sy*j + sm*c + naux*sm*p (include/safara.h)."""
+    return torch.empty((nplanes, naux, ny, pitch(nx)), dtype=torch.float64, device=device)
+
+
+def unpack_aux(t: torch.Tensor, nx: int) -> np.ndarray:
+    """Canonical (nz, naux, ny, sy) -> logical (nz, ny, nx, naux)."""
+    return np.ascontiguousarray(t[..., :nx].permute(0, 2, 3, 1).cpu().numpy())
+
+
+def rhs_aux(u: torch.Tensor, forcing: torch.Tensor, out: torch.Tensor, aux: torch.Tensor,
+            nx: int, coeffs: Coeffs, strict: bool = False, stream=None,
+            dims: Dims | None = None) -> torch.Tensor:
+    """compute_rhs pass that also writes the step-0 fields into ``aux``
+    (naux = aux.shape[1] for canonical tensors: 6 BT or 7 with SP speed)."""
+    for t, n in ((u, "u"), (forcing, "forcing"), (out, "out"), (aux, "aux")):
+        _check_field(t, n)
+    if dims is None:
+        nz, _, ny, _ = u.shape
+        dims = canonical_dims(nx, ny, nz)
+    naux = int(aux.shape[1]) if aux.dim() == 4 else SAFARA_AUX_BT
+    flags = SAFARA_FLAG_STRICT if strict else 0
+    check(lib().safara_rhs_aux(u.data_ptr(), forcing.data_ptr(), out.data_ptr(), aux.data_ptr(),
+                               naux, ctypes.byref(dims), ctypes.byref(coeffs), flags,
+                               _stream_ptr(stream)), "safara_rhs_aux")
+    return aux
+
+
+def rhs_slab_aux(u_slab, forcing_slab, out_slab, aux_slab, nx: int, nz: int, k0: int,
+                 coeffs: Coeffs, part: int = SAFARA_PART_ALL, strict: bool = False,
+                 stream=None) -> torch.Tensor:
+    for t, n in ((u_slab, "u_slab"), (forcing_slab, "forcing_slab"), (out_slab, "out_slab"),
+                 (aux_slab, "aux_slab")):
+        _check_field(t, n)
+    nzl, _, ny, _ = forcing_slab.shape
+    dims = canonical_dims(nx, ny, nz)
+    flags = SAFARA_FLAG_STRICT if strict else 0
+    check(lib().safara_rhs_slab_aux(u_slab.data_ptr(), forcing_slab.data_ptr(),
+                                    out_slab.data_ptr(), aux_slab.data_ptr(),
+                                    int(aux_slab.shape[1]), ctypes.byref(dims), int(k0), int(nzl),
+                                    ctypes.byref(coeffs), flags, int(part), _stream_ptr(stream)),
+          "safara_rhs_slab_aux")
+    return aux_slab
+
+
+_norm_work: dict[int, torch.Tensor] = {}
+
+
+def rhs_sumsq(r: torch.Tensor, nx: int, nz: int | None = None, k0: int = 0, stream=None,
+              out: torch.Tensor | None = None, dims: Dims | None = None) -> torch.Tensor:
+    """Per-component sums of rhs^2 over the interior points of the planes
+    ``r`` holds (plane p = global k0+p); a 5-element device tensor (async)."""
+    _check_field(r, "rhs")
+    nzl, _, ny, _ = r.shape
+    nz = nzl if nz is None else nz
+    if dims is None:
+        dims = canonical_dims(nx, ny, nz)
+    dev = r.device.index if r.device.index is not None else torch.cuda.current_device()
+    work = _norm_work.get(dev)
+    if work is None:
+        work = torch.empty(lib().safara_norm_work_doubles(), dtype=torch.float64, device=r.device)
+        _norm_work[dev] = work
+    if out is None:
+        out = torch.empty(5, dtype=torch.float64, device=r.device)
+    check(lib().safara_rhs_sumsq(r.data_ptr(), ctypes.byref(dims), int(k0), int(nzl),
+                                 work.data_ptr(), out.data_ptr(), _stream_ptr(stream)),
+          "safara_rhs_sumsq")
+    return out
+
+
+def rhs_norm(r: torch.Tensor, nx: int, stream=None) -> np.ndarray:
+    """NPB rhs_norm of a full-grid canonical rhs: sqrt(sum rhs(m)^2 /
+    ((nx-2)(ny-2)(nz-2))) per component (host numpy, synchronises)."""
+    nz, _, ny, _ = r.shape
+    s = rhs_sumsq(r, nx, stream=stream).cpu().numpy()
+    return np.sqrt(s / ((nx - 2) * (ny - 2) * (nz - 2)))
