@@ -44,6 +44,11 @@ def parse():
     ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--e2e-chunks", type=int, default=8,
                     help="k-chunks of the pipelined H2D / compute / D2H e2e path")
+    ap.add_argument("--workload", default="rhs", choices=["rhs", "rhs_aux", "seismic_dz"],
+                    help="rhs: the headline compute_rhs pass; rhs_aux: the same pass also "
+                         "writing the 6 step-0 fields (SURVEY §8(f) f1); seismic_dz: the "
+                         "PAPER.md Fig. 8 loop (f4) on --seismic-n^3")
+    ap.add_argument("--seismic-n", type=int, default=256)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--soak-s", type=float, default=1.0,
                     help="untimed passes before the timed region so the clock sampler "
@@ -222,9 +227,16 @@ def run_single(args):
     dr = torch.empty_like(du)
     stream = torch.cuda.current_stream()
     pts = nx * ny * nz
+    bytes_per_point = BYTES_PER_POINT
+    if args.workload == "rhs_aux":
+        da = sr.empty_aux(nx, ny, nz, sr.SAFARA_AUX_BT)
+        bytes_per_point += 8 * sr.SAFARA_AUX_BT
 
-    def step():
-        sr.rhs(du, df, dr, nx, c, strict=args.strict, stream=stream)
+        def step():
+            sr.rhs_aux(du, df, dr, da, nx, c, strict=args.strict, stream=stream)
+    else:
+        def step():
+            sr.rhs(du, df, dr, nx, c, strict=args.strict, stream=stream)
 
     for _ in range(max(args.warmup, 3)):
         step()
@@ -256,14 +268,14 @@ def run_single(args):
     ms_per_step = total_ms / args.steps
     value = pts / (ms_per_step * 1e-3) / 1e9
     kern_ms = sum(per) / len(per)
-    achieved = BYTES_PER_POINT * pts / (kern_ms * 1e-3) / 1e9
+    achieved = bytes_per_point * pts / (kern_ms * 1e-3) / 1e9
     peak, peak_kind = measured_peaks()
     key = f"{bench}-{cls}"
     traffic = ncu_traffic(key)
 
     # e2e: host (pinned) buffers through the C ABI, H2D + pass + D2H per step
     e2e_ms, nbytes = float("nan"), 0
-    if args.e2e_steps > 0:
+    if args.e2e_steps > 0 and args.workload == "rhs":
         hu, hf = sr.pack(inp.u, pin=True), sr.pack(inp.forcing, pin=True)
         hr = torch.empty(hu.shape, dtype=torch.float64).pin_memory()
         for _ in range(2):
@@ -292,7 +304,7 @@ def run_single(args):
         "hbm_gbs": achieved,
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "peak_kind": peak_kind, "traffic": traffic,
-                     "bytes_per_point": BYTES_PER_POINT, "kernel_ms": kern_ms,
+                     "bytes_per_point": bytes_per_point, "kernel_ms": kern_ms,
                      "frac_of_8000": achieved / 8000.0},
         "clocks": clocks,
         "e2e": {"value": pts / (e2e_ms * 1e-3) / 1e9, "unit": "Gpt/s",
@@ -306,8 +318,66 @@ def run_single(args):
     print(json.dumps(line), flush=True)
 
 
+def run_seismic(args):
+    """PAPER.md Fig. 8 dz loop: 3 inputs + 1 output of
+    n^3 doubles, 32 algorithmic bytes per point (HBM-bound)."""
+    import numpy as np
+    import torch
+
+    import paper_conf_icpp_tiankexc16_b200 as sr
+
+    torch.cuda.set_device(0)
+    sr.init(0)
+    n = args.seismic_n
+    sy = sr.pitch(n)
+    g = torch.Generator(device="cuda").manual_seed(1)
+    vz = [torch.randn((n, n, sy), dtype=torch.float64, device="cuda", generator=g)
+          for _ in range(3)]
+    out = torch.zeros_like(vz[0])
+    stream = torch.cuda.current_stream()
+    pts = (n - 1) ** 3  # written points
+    for _ in range(max(args.warmup, 3)):
+        sr.seismic_dz(*vz, out, 0.01, n, stream=stream)
+    sampler = ClockSampler(0)
+    sampler.start()
+    t_end = time.time() + args.soak_s
+    while time.time() < t_end:
+        for _ in range(20):
+            sr.seismic_dz(*vz, out, 0.01, n, stream=stream)
+        torch.cuda.synchronize()
+    ev = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps + 1)]
+    l0 = sr.launch_count()
+    torch.cuda.synchronize()
+    ev[0].record(stream)
+    for k in range(args.steps):
+        sr.seismic_dz(*vz, out, 0.01, n, stream=stream)
+        ev[k + 1].record(stream)
+    torch.cuda.synchronize()
+    per = [ev[k].elapsed_time(ev[k + 1]) for k in range(args.steps)]
+    clocks = ClockSampler.summarise(sampler.stop())
+    ms = ev[0].elapsed_time(ev[-1]) / args.steps
+    kern_ms = float(np.mean(per))
+    peak, peak_kind = measured_peaks()
+    achieved = 32 * pts / (kern_ms * 1e-3) / 1e9
+    print(json.dumps({
+        "metric": "seismic dz grid-points/s", "value": pts / (ms * 1e-3) / 1e9, "unit": "Gpt/s",
+        "n_gpus": 1, "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms,
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
+        "data": "synthetic",
+        "config": {"workload": f"355.seismic dz loop (PAPER.md Fig. 8) {n}^3 fp64",
+                   "grid": [n, n, n], "points": pts,
+                   "l2": f"4 x {n * n * sy * 8 / 1e6:.0f} MB > 126 MB L2, no flush"},
+        "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                     "frac": achieved / peak, "peak_kind": peak_kind, "traffic": None,
+                     "bytes_per_point": 32, "kernel_ms": kern_ms},
+        "clocks": clocks, "gpu_launches": sr.launch_count() - l0}), flush=True)
+
+
 def main():
     args = parse()
+    if args.workload == "seismic_dz" and args.impl != "reference":
+        run_seismic(args)
+        return
     if args.impl == "reference":
         run_reference(args)
         return

@@ -175,6 +175,30 @@ int safara_norm_work_doubles(void);
 int safara_rhs_sumsq(const double *rhs, const safara_dims_t *dims, int k0,
                      int nzl, double *work, double *out, void *stream);
 
+/* ---- the 355.seismic dz loop (Fig. 8) -----
+ *
+ * The loop nest the paper uses to motivate `dim` and `small` (L1078-1096):
+ *   for j in [1, ny-1], i in [0, nx-2] (parallel), k in [1, nz-1] (seq):
+ *     value_dz(i,j,k) = ((vz1(k) - vz1(k-1))/h + (vz2(k) - vz2(k-1))/h)
+ *                       + (vz3(k) - vz3(k-1))/h          (at (i, j))
+ * i.e. Fig. 8's 1-based ranges j = 2..ny, i = 1..nx-1, k = 2..nz with zero
+ * lower bounds.  value_dz is written at exactly those points (the others are
+ * left untouched).  All four arrays share ONE descriptor (`dim`, the
+ * "(0:NX,0:NY,0:NZ)" form of L1194-1202): element (i, j, k) at
+ * i + sy*j + sk*k, offsets 32-bit (`small`).  IEEE division, evaluated as
+ * written (bit-identical to the oracle).
+ * Errors: SAFARA_ERR_ARG (NULL, h zero or not finite, value_dz overlapping an
+ * input), SAFARA_ERR_SHAPE (extent < 2), SAFARA_ERR_LAYOUT (sy < nx or
+ * sk < sy*ny), SAFARA_ERR_ALIGN (pointer not 8-byte aligned),
+ * SAFARA_ERR_TOO_LARGE (offset >= 2^31).  Asynchronous; one kernel launch. */
+typedef struct {
+    int32_t nx, ny, nz;
+    int32_t sy, sk;
+} safara_dims3_t;
+int safara_seismic_dz(const double *vz1, const double *vz2, const double *vz3,
+                      double *value_dz, const safara_dims3_t *dims, double h,
+                      void *stream);
+
 /* End-to-end call with HOST arrays (canonical layout): copies u and forcing
  * host->device into the caller's device buffers u_dev/forcing_dev, runs the
  * pass into rhs_dev and copies rhs device->host.  The grid is cut into

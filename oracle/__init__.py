@@ -82,6 +82,8 @@ def _load():
             lib.oracle_compute_aux.restype = ctypes.c_int
             lib.oracle_rhs_sumsq.argtypes = [ctypes.c_int] * 3 + [dp, dp]
             lib.oracle_rhs_sumsq.restype = ctypes.c_int
+            lib.oracle_seismic_dz.argtypes = [ctypes.c_int] * 3 + [dp] * 4 + [ctypes.c_double]
+            lib.oracle_seismic_dz.restype = ctypes.c_int
             _lib = lib
     return _lib
 
@@ -166,4 +168,20 @@ def rhs_sumsq(rhs: np.ndarray) -> np.ndarray:
     dp = ctypes.POINTER(ctypes.c_double)
     if _load().oracle_rhs_sumsq(nx, ny, nz, rn.ctypes.data_as(dp), out.ctypes.data_as(dp)) != 0:
         raise ValueError("oracle_rhs_sumsq: extents must be >= 3")
+    return out
+
+
+def seismic_dz(vz1: np.ndarray, vz2: np.ndarray, vz3: np.ndarray, h: float,
+               init: np.ndarray | None = None) -> np.ndarray:
+    """PAPER.md Fig. 8 dz loop.  Arrays are indexed
+    [k, j, i] (C order of Fortran vz(i,j,k)); points outside the loop ranges
+    keep ``init`` (default NaN)."""
+    nz, ny, nx = vz1.shape
+    out = (np.full((nz, ny, nx), np.nan) if init is None
+           else np.array(init, dtype=np.float64, copy=True))
+    a = [np.ascontiguousarray(v, dtype=np.float64) for v in (vz1, vz2, vz3)]
+    dp = ctypes.POINTER(ctypes.c_double)
+    if _load().oracle_seismic_dz(nx, ny, nz, *(v.ctypes.data_as(dp) for v in a),
+                                 out.ctypes.data_as(dp), float(h)) != 0:
+        raise ValueError("oracle_seismic_dz: extents must be >= 2")
     return out

@@ -71,4 +71,9 @@ int oracle_compute_aux(int nx, int ny, int nz, const oracle_consts_t *c,
  * rhs(m)^2 (k, j, i loop order).  Returns 0 or -1. */
 int oracle_rhs_sumsq(int nx, int ny, int nz, const double *rhs, double *out);
 
+/* 355.seismic dz loop of PAPER.md Fig. 8 (zero lower bounds; see .c).
+ * Dense Fortran-order arrays vz(i,j,k) at i + nx*(j + ny*k).  Returns 0/-1. */
+int oracle_seismic_dz(int nx, int ny, int nz, const double *vz_1, const double *vz_2,
+                      const double *vz_3, double *value_dz, double h);
+
 #endif

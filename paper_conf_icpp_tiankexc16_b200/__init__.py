@@ -5,14 +5,15 @@ this package only marshals torch tensors into that ABI.  PyTorch supplies
 device memory, streams and process groups.  See DESIGN.md.
 """
 from ._abi import (SAFARA_AUX_BT, SAFARA_AUX_SP, SAFARA_FLAG_STRICT, SAFARA_PART_ALL,
-                   SAFARA_PART_EDGE, SAFARA_PART_INTERIOR, Coeffs, Dims, SafaraError)
+                   SAFARA_PART_EDGE, SAFARA_PART_INTERIOR, Coeffs, Dims, Dims3, SafaraError)
 from .rhs import (AUX_NAMES, canonical_dims, coeffs_nas, empty_aux, empty_field, init,
                   kernel_info, launch_count, pack, pitch, rhs, rhs_aux, rhs_host, rhs_norm,
-                  rhs_slab, rhs_slab_aux, rhs_sumsq, unpack, unpack_aux, validate_dims)
+                  rhs_slab, rhs_slab_aux, rhs_sumsq, seismic_dz, unpack, unpack_aux,
+                  validate_dims)
 
 __all__ = [
     "AUX_NAMES", "SAFARA_AUX_BT", "SAFARA_AUX_SP", "empty_aux", "rhs_aux", "rhs_norm",
-    "rhs_slab_aux", "rhs_sumsq", "unpack_aux",
+    "rhs_slab_aux", "rhs_sumsq", "unpack_aux", "seismic_dz",
     "SAFARA_FLAG_STRICT", "SAFARA_PART_ALL", "SAFARA_PART_EDGE", "SAFARA_PART_INTERIOR",
     "Coeffs", "Dims", "SafaraError", "canonical_dims", "coeffs_nas", "empty_field", "init",
     "kernel_info", "launch_count", "pack", "pitch", "rhs", "rhs_host", "rhs_slab", "unpack",

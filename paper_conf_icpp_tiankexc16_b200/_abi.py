@@ -37,6 +37,11 @@ class Coeffs(ctypes.Structure):
         (n, ctypes.c_double * 5) for n in ("dxt", "dyt", "dzt", "xxcon", "yycon", "zzcon")]
 
 
+class Dims3(ctypes.Structure):
+    """safara_dims3_t: the shared 3-D descriptor of the seismic dz loop."""
+    _fields_ = [(n, ctypes.c_int32) for n in ("nx", "ny", "nz", "sy", "sk")]
+
+
 class KernelInfo(ctypes.Structure):
     _fields_ = [(n, ctypes.c_int) for n in
                 ("regs_per_thread", "local_bytes", "smem_bytes", "threads_per_cta",
@@ -68,6 +73,7 @@ _SIGS = {
     "safara_norm_work_doubles": ([], ctypes.c_int),
     "safara_rhs_sumsq": ([_dp, ctypes.POINTER(Dims), ctypes.c_int, ctypes.c_int, _dp, _dp, _dp],
                          ctypes.c_int),
+    "safara_seismic_dz": ([_dp] * 4 + [ctypes.POINTER(Dims3), ctypes.c_double, _dp], ctypes.c_int),
     "safara_launch_count": ([], ctypes.c_int64),
     "safara_kernel_info": ([ctypes.c_int, ctypes.POINTER(KernelInfo)], ctypes.c_int),
     "safara_strerror": ([ctypes.c_int], ctypes.c_char_p),

@@ -27,6 +27,7 @@ UNITS = [
     ("rhs_fast.cu", ["--fmad=true", "-Xptxas", "-v"]),
     ("rhs_strict.cu", ["--fmad=false", "-Xptxas", "-v"]),
     ("norm.cu", []),
+    ("seismic.cu", ["-Xptxas", "-v"]),
     ("api.cu", []),
 ]
 DEPS = ["rhs_kernel.cuh", "rhs_variant.inc", "safara_internal.h"]

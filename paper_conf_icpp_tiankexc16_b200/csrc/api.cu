@@ -228,8 +228,11 @@ int launch(const double *u, const double *f, double *r, const safara_dims_t &d, 
         ncta = std::min<long long>(max_ctas, 16);
     }
     p.ncta = (int)ncta;
-    // SMs the compute grid leaves idle take the boundary faces
-    p.nface_cta = (g_tune.face_ctas && fk_hi > fk_lo && p.units > 0 && ncta < max_ctas)
+    // SMs the compute grid leaves idle take the boundary faces -- unless the
+    // aux fields are requested: then each face point also reads u and writes
+    // naux strided values, too much for a handful of SMs, so every compute
+    // CTA takes a share before its march
+    p.nface_cta = (g_tune.face_ctas && !aux && fk_hi > fk_lo && p.units > 0 && ncta < max_ctas)
                       ? (int)std::min<long long>(max_ctas - ncta, 32) : 0;
 
 #ifdef SAFARA_TIMELINE
@@ -569,6 +572,32 @@ int safara_rhs_sumsq(const double *rhs, const safara_dims_t *dims, int k0, int n
                                  nk, work, out, (cudaStream_t)stream);
     if (e != cudaSuccess) return SAFARA_ERR_CUDA;
     g_launches.fetch_add(2, std::memory_order_relaxed);
+    return SAFARA_OK;
+}
+
+int safara_seismic_dz(const double *vz1, const double *vz2, const double *vz3, double *value_dz,
+                      const safara_dims3_t *dims, double h, void *stream) {
+    int dev;
+    int rc = current_device(&dev);
+    if (rc) return rc;
+    if (!dims || !vz1 || !vz2 || !vz3 || !value_dz) return SAFARA_ERR_ARG;
+    if (!(h != 0.0) || h - h != 0.0) return SAFARA_ERR_ARG;  // zero, NaN or infinite
+    const safara_dims3_t &d = *dims;
+    if (d.nx < 2 || d.ny < 2 || d.nz < 2) return SAFARA_ERR_SHAPE;
+    if (d.sy < d.nx || d.sk < (long long)d.sy * d.ny) return SAFARA_ERR_LAYOUT;
+    const long long maxo = (long long)(d.nx - 1) + (long long)d.sy * (d.ny - 1) +
+                           (long long)d.sk * (d.nz - 1);
+    if (maxo >= (1LL << 31)) return SAFARA_ERR_TOO_LARGE;  // `small`
+    if (((uintptr_t)vz1 | (uintptr_t)vz2 | (uintptr_t)vz3 | (uintptr_t)value_dz) & 7u)
+        return SAFARA_ERR_ALIGN;
+    const long long bytes = (maxo + 1) * (long long)sizeof(double);
+    if (overlaps(value_dz, bytes, vz1, bytes) || overlaps(value_dz, bytes, vz2, bytes) ||
+        overlaps(value_dz, bytes, vz3, bytes))
+        return SAFARA_ERR_ARG;
+    cudaError_t e = launch_seismic_dz(vz1, vz2, vz3, value_dz, d.nx, d.ny, d.nz, d.sy, d.sk, h,
+                                      g_dev[dev].sms, (cudaStream_t)stream);
+    if (e != cudaSuccess) return SAFARA_ERR_CUDA;
+    g_launches.fetch_add(1, std::memory_order_relaxed);
     return SAFARA_OK;
 }
 

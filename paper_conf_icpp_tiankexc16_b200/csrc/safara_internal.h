@@ -95,6 +95,11 @@ int norm_grid();
 cudaError_t launch_sumsq(const double *rhs, int nx, int ny, int sy, int sm, int sk, int kl0, int nk,
                          double *work, double *out, cudaStream_t s);
 
+// seismic.cu: PAPER.md Fig. 8 dz loop (f4)
+cudaError_t launch_seismic_dz(const double *vz1, const double *vz2, const double *vz3, double *out,
+                              int nx, int ny, int nz, int sy, int sk, double h, int sms,
+                              cudaStream_t s);
+
 // attr: 4 entries (production NAS path, general coefficients, aux, NAS + aux)
 cudaError_t setup_rhs_fast(int *ctas_per_sm, cudaFuncAttributes *attr);
 cudaError_t setup_rhs_strict(int *ctas_per_sm, cudaFuncAttributes *attr);

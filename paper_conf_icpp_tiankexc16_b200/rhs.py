@@ -14,7 +14,7 @@ import numpy as np
 import torch
 
 from ._abi import (SAFARA_AUX_BT, SAFARA_AUX_SP, SAFARA_FLAG_STRICT, SAFARA_PART_ALL, Coeffs,
-                   Dims, KernelInfo, check, lib)
+                   Dims, Dims3, KernelInfo, check, lib)
 
 _initialised: set[int] = set()
 
@@ -225,3 +225,22 @@ def rhs_norm(r: torch.Tensor, nx: int, stream=None) -> np.ndarray:
     nz, _, ny, _ = r.shape
     s = rhs_sumsq(r, nx, stream=stream).cpu().numpy()
     return np.sqrt(s / ((nx - 2) * (ny - 2) * (nz - 2)))
+
+
+# ---- the 355.seismic dz loop (Fig. 8) --------
+
+def seismic_dz(vz1: torch.Tensor, vz2: torch.Tensor, vz3: torch.Tensor, out: torch.Tensor,
+               h: float, nx: int, stream=None) -> torch.Tensor:
+    """value_dz of Fig. 8 into ``out`` for (nz, ny, sy) float64 CUDA tensors
+    sharing one pitched layout (sy >= nx): j in [1, ny-1], i in [0, nx-2],
+    k in [1, nz-1]; other points untouched."""
+    for t, n in ((vz1, "vz1"), (vz2, "vz2"), (vz3, "vz3"), (out, "value_dz")):
+        _check_field(t, n)
+        if t.shape != vz1.shape or t.dim() != 3:
+            raise ValueError("vz1, vz2, vz3 and value_dz must share one (nz, ny, sy) shape")
+    nz, ny, sy = vz1.shape
+    d = Dims3(nx, ny, nz, sy, sy * ny)
+    check(lib().safara_seismic_dz(vz1.data_ptr(), vz2.data_ptr(), vz3.data_ptr(), out.data_ptr(),
+                                  ctypes.byref(d), float(h), _stream_ptr(stream)),
+          "safara_seismic_dz")
+    return out
