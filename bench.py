@@ -50,6 +50,9 @@ def parse():
                          "PAPER.md Fig. 8 loop (f4) on --seismic-n^3")
     ap.add_argument("--seismic-n", type=int, default=256)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--launch-events", action="store_true",
+                    help="record an event after every launch (diagnostic; an event between "
+                         "launches also serialises programmatic dependent launch)")
     ap.add_argument("--soak-s", type=float, default=1.0,
                     help="untimed passes before the timed region so the clock sampler "
                          "sees the GPU under load")
@@ -257,11 +260,16 @@ def run_single(args):
     ev[0].record(stream)
     for k in range(args.steps):
         step()
-        ev[k + 1].record(stream)
+        if args.launch_events:
+            ev[k + 1].record(stream)
+    if not args.launch_events:
+        ev[-1].record(stream)
     torch.cuda.synchronize()
     launches = sr.launch_count() - l0
-    per = [ev[k].elapsed_time(ev[k + 1]) for k in range(args.steps)]
     total_ms = ev[0].elapsed_time(ev[-1])
+    # one launch per step: the average launch duration is the step time
+    per = ([ev[k].elapsed_time(ev[k + 1]) for k in range(args.steps)] if args.launch_events
+           else [total_ms / args.steps])
     rows = sampler.stop()
     clocks = ClockSampler.summarise(rows)
 

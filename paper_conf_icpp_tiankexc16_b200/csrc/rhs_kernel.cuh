@@ -58,6 +58,9 @@
 #ifndef SAFARA_PROBE
 #define SAFARA_PROBE 0  // roofline probes: 1 memory only, 2 compute only (no TMA waits/refills, no stores), 3 no rhs stores
 #endif
+#ifndef SAFARA_PDL
+#define SAFARA_PDL 0  // programmatic dependent launch (see launch_pdl; A/B on B200: no gain, profiles/ab_pdl_r01.txt)
+#endif
 #ifndef SAFARA_STORE
 #define SAFARA_STORE 0  // rhs stores: 0 st.global.cs, 1 default caching, 2 none (probe)
 #endif
@@ -154,6 +157,20 @@ __device__ __forceinline__ void tma_prefetch_l2_4d(const CUtensorMap *map, int c
             reinterpret_cast<uint64_t>(map)),
         "r"(c0), "r"(c1), "r"(c2), "r"(c3)
         : "memory");
+}
+
+// PDL: let the next grid on the stream be scheduled (its CTAs take SMs as
+// ours exit and park in grid_dep_wait), and wait for the previous grid's
+// completion before this grid's first global access.
+__device__ __forceinline__ void grid_dep_launch() {
+#if SAFARA_PDL
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+#endif
+}
+__device__ __forceinline__ void grid_dep_wait() {
+#if SAFARA_PDL
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+#endif
 }
 
 __device__ __forceinline__ void prefetch_tmap(const CUtensorMap *map) {
@@ -839,7 +856,9 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensor
 #endif
     // Extra CTAs beyond the compute grid (on SMs the lockstep schedule leaves
     // idle) only copy the boundary faces.
+    grid_dep_launch();
     if ((int)blockIdx.x >= P.ncta) {
+        grid_dep_wait();
         copy_faces<AUX>(P, (int)blockIdx.x - P.ncta, P.nface_cta);
 #ifdef SAFARA_TIMELINE
         if (threadIdx.x == 0 && P.dbg) {
@@ -868,6 +887,7 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensor
         fence_mbar_init();
     }
     __syncthreads();
+    grid_dep_wait();
 
     int ub, ue;
     if (P.parts > 0) {
