@@ -131,6 +131,77 @@ int safara_rhs_slab(const double *u_slab, const double *forcing_slab,
                     int nzl, const safara_coeffs_t *coeffs, int flags,
                     int part, void *stream);
 
+/* ---- the halo fused into the pass (peer memory) --------
+ *
+ * The z-slab pass of safara_rhs_slab (PART_ALL) without a separate halo
+ * exchange: the only values a slab needs from its neighbours are the OWN
+ * (i, j) columns of the two planes beyond each slab end (the zeta window,
+ * SURVEY App. A steps 6-7; xi/eta stencils stay in-plane), so the kernel
+ * loads them directly from the neighbours' u slabs through peer pointers
+ * (NVLink load/store access; CUDA IPC mappings, see safara_ipc_*), one
+ * launch per pass and no exchange step.  Ghost planes of u_slab are neither
+ * read nor written.
+ *   u_lo / u_hi:  the lower / upper neighbour's u slab in the safara_rhs_slab
+ *                 layout (its local plane p = global k0_lo - 2 + p, resp.
+ *                 k0_hi - 2 + p), same descriptor; NULL iff there is no
+ *                 neighbour on that side (k0 == 0, resp. k0 + nzl == nz).
+ *                 Only its owned planes k0-2, k0-1 (resp. k0+nzl, k0+nzl+1)
+ *                 are read, so the neighbour must own >= 2 planes.
+ *   flags:        this rank's SAFARA_PEER_WORDS uint64 words (device memory,
+ *                 zeroed once before the first epoch); flags_lo / flags_hi
+ *                 the neighbours' (peer pointers), NULL iff u_lo / u_hi is.
+ *   epoch:        0 = no synchronisation (the caller guarantees the
+ *                 neighbours' u is final and unchanged while any rank runs,
+ *                 e.g. a static benchmark input); > 0 = the pass number,
+ *                 strictly increasing across calls and equal on neighbouring
+ *                 ranks.  With epoch > 0 every CTA first publishes "my u of
+ *                 this epoch is final" (release store into the neighbours'
+ *                 READY words), readers acquire the neighbour's READY word
+ *                 before their peer loads, and the grid does not complete
+ *                 until both neighbours have finished reading this rank's u
+ *                 (their DONE words), so the caller may overwrite u after
+ *                 the pass in stream order -- the contract of a halo exchange
+ *                 without one.  A wait longer than ~2 s gives up and
+ *                 increments flags[SAFARA_PEER_TIMEOUTS] (results are then
+ *                 undefined; nothing hangs).
+ * Results are bit-identical to safara_rhs_slab (same kernel body).
+ * Errors: those of safara_rhs_slab, plus SAFARA_ERR_ARG (peer NULL, a
+ * neighbour pointer missing / present against the grid ends, flags NULL or
+ * not 8-byte aligned with epoch > 0, k0_lo / k0_hi inconsistent).          */
+#define SAFARA_PEER_LO_READY 0  /* written by the lower neighbour           */
+#define SAFARA_PEER_HI_READY 1  /* written by the upper neighbour           */
+#define SAFARA_PEER_LO_DONE  2  /* lower neighbour finished reading our u   */
+#define SAFARA_PEER_HI_DONE  3  /* upper neighbour finished reading our u   */
+#define SAFARA_PEER_ARRIVED  4  /* own grid's CTA arrival counter           */
+#define SAFARA_PEER_TIMEOUTS 5  /* waits that gave up (should stay 0)       */
+#define SAFARA_PEER_TIMEOUT_WORDS 6  /* bit w set: a wait on word w gave up */
+#define SAFARA_PEER_WORDS    8
+typedef struct {
+    const double *u_lo, *u_hi;      /* neighbours' u slabs (peer pointers)   */
+    int32_t k0_lo, k0_hi;           /* neighbours' first owned global plane  */
+    uint64_t *flags;                /* this rank's flag words                */
+    uint64_t *flags_lo, *flags_hi;  /* neighbours' flag words (peer)         */
+    uint64_t epoch;
+} safara_peer_t;
+int safara_rhs_peer(const double *u_slab, const double *forcing_slab,
+                    double *rhs_slab, const safara_dims_t *dims, int k0,
+                    int nzl, const safara_peer_t *peer,
+                    const safara_coeffs_t *coeffs, int flags, void *stream);
+
+/* CUDA IPC plumbing for the peer pointers (host calls, synchronous).
+ *   safara_ipc_get: export the allocation holding device pointer dptr:
+ *     handle <- SAFARA_IPC_HANDLE_BYTES opaque bytes, *offset <- dptr minus
+ *     the allocation base.  SAFARA_ERR_ARG (NULL), SAFARA_ERR_CUDA (not an
+ *     IPC-exportable cudaMalloc allocation, e.g. a VMM/expandable segment).
+ *   safara_ipc_open: map another process's export on the current device
+ *     (peer access enabled lazily); *dptr <- mapped base + offset.
+ *   safara_ipc_close: unmap a pointer returned by safara_ipc_open (pass the
+ *     same offset).                                                         */
+#define SAFARA_IPC_HANDLE_BYTES 64
+int safara_ipc_get(const void *dptr, void *handle, int64_t *offset);
+int safara_ipc_open(const void *handle, int64_t offset, void **dptr);
+int safara_ipc_close(void *dptr, int64_t offset);
+
 /* ---- the step-0 auxiliary fields and the rhs norm ------
  *
  * NAS compute_rhs forms, in its step 0, the per-point fields

@@ -5,9 +5,10 @@ this package only marshals torch tensors into that ABI.  PyTorch supplies
 device memory, streams and process groups.  See DESIGN.md.
 """
 from ._abi import (SAFARA_AUX_BT, SAFARA_AUX_SP, SAFARA_FLAG_STRICT, SAFARA_PART_ALL,
-                   SAFARA_PART_EDGE, SAFARA_PART_INTERIOR, Coeffs, Dims, Dims3, SafaraError)
+                   SAFARA_PART_EDGE, SAFARA_PART_INTERIOR, Coeffs, Dims, Dims3, Peer, SafaraError)
 from .rhs import (AUX_NAMES, canonical_dims, coeffs_nas, empty_aux, empty_field, init,
-                  kernel_info, launch_count, pack, pitch, rhs, rhs_aux, rhs_host, rhs_norm,
+                  ipc_close, ipc_get, ipc_open, kernel_info, launch_count, pack, pitch, rhs,
+                  rhs_aux, rhs_host, rhs_norm, rhs_peer,
                   rhs_slab, rhs_slab_aux, rhs_sumsq, seismic_dz, unpack, unpack_aux,
                   validate_dims)
 
@@ -17,5 +18,5 @@ __all__ = [
     "SAFARA_FLAG_STRICT", "SAFARA_PART_ALL", "SAFARA_PART_EDGE", "SAFARA_PART_INTERIOR",
     "Coeffs", "Dims", "SafaraError", "canonical_dims", "coeffs_nas", "empty_field", "init",
     "kernel_info", "launch_count", "pack", "pitch", "rhs", "rhs_host", "rhs_slab", "unpack",
-    "validate_dims",
+    "validate_dims", "Peer", "rhs_peer", "ipc_get", "ipc_open", "ipc_close",
 ]

@@ -48,6 +48,19 @@ class KernelInfo(ctypes.Structure):
                  "ctas_per_sm", "tile_x", "tile_y", "stages")]
 
 
+class Peer(ctypes.Structure):
+    """safara_peer_t."""
+    _fields_ = [("u_lo", ctypes.c_void_p), ("u_hi", ctypes.c_void_p),
+                ("k0_lo", ctypes.c_int32), ("k0_hi", ctypes.c_int32),
+                ("flags", ctypes.c_void_p), ("flags_lo", ctypes.c_void_p),
+                ("flags_hi", ctypes.c_void_p), ("epoch", ctypes.c_uint64)]
+
+
+SAFARA_PEER_WORDS = 8
+SAFARA_PEER_LO_READY, SAFARA_PEER_HI_READY, SAFARA_PEER_LO_DONE, SAFARA_PEER_HI_DONE = 0, 1, 2, 3
+SAFARA_PEER_ARRIVED, SAFARA_PEER_TIMEOUTS = 4, 5
+SAFARA_IPC_HANDLE_BYTES = 64
+
 _lock = threading.Lock()
 _lib = None
 
@@ -70,6 +83,13 @@ _SIGS = {
     "safara_rhs_slab_aux": ([_dp, _dp, _dp, _dp, ctypes.c_int, ctypes.POINTER(Dims), ctypes.c_int,
                              ctypes.c_int, ctypes.POINTER(Coeffs), ctypes.c_int, ctypes.c_int, _dp],
                             ctypes.c_int),
+    "safara_rhs_peer": ([_dp, _dp, _dp, ctypes.POINTER(Dims), ctypes.c_int, ctypes.c_int,
+                         ctypes.POINTER(Peer), ctypes.POINTER(Coeffs), ctypes.c_int, _dp],
+                        ctypes.c_int),
+    "safara_ipc_get": ([_dp, ctypes.c_char_p, ctypes.POINTER(ctypes.c_int64)], ctypes.c_int),
+    "safara_ipc_open": ([ctypes.c_char_p, ctypes.c_int64, ctypes.POINTER(ctypes.c_void_p)],
+                        ctypes.c_int),
+    "safara_ipc_close": ([_dp, ctypes.c_int64], ctypes.c_int),
     "safara_norm_work_doubles": ([], ctypes.c_int),
     "safara_rhs_sumsq": ([_dp, ctypes.POINTER(Dims), ctypes.c_int, ctypes.c_int, _dp, _dp, _dp],
                          ctypes.c_int),

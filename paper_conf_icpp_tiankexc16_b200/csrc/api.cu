@@ -161,6 +161,14 @@ int encode_map(CUtensorMap *map, const double *base, const safara_dims_t &d, int
     return r == CUDA_SUCCESS ? SAFARA_OK : SAFARA_ERR_CUDA;
 }
 
+// f2 (safara_rhs_peer): where the planes beyond the slab come from.
+struct PeerCfg {
+    int pk_lo, pk_hi, lo_koff, hi_koff;
+    const double *u_lo, *u_hi;
+    unsigned long long *flags, *flags_lo, *flags_hi;
+    unsigned long long epoch;
+};
+
 // Shared launch path.  u has nzu planes, u plane = k - k0 + ukoff; forcing
 // and rhs start at global plane k0.  [ka0,kb0) U [ka1,kb1) are computed;
 // boundary faces of local planes [fk_lo, fk_hi) are copied.
@@ -168,7 +176,7 @@ int launch(const double *u, const double *f, double *r, const safara_dims_t &d, 
            int k0,
            int ukoff, int ka0, int kb0, int ka1, int kb1, int fk_lo, int fk_hi,
            const safara_coeffs_t *coeffs, int flags, cudaStream_t stream,
-           double *aux = nullptr, int naux = 0, int ska = 0) {
+           double *aux = nullptr, int naux = 0, int ska = 0, const PeerCfg *peer = nullptr) {
     int dev;
     int rc = current_device(&dev);
     if (rc) return rc;
@@ -201,6 +209,15 @@ int launch(const double *u, const double *f, double *r, const safara_dims_t &d, 
     p.fk_lo = fk_lo; p.fk_hi = fk_hi;
     p.u = u; p.f = f; p.r = r;
     p.aux = aux; p.naux = naux; p.ska = ska;
+    p.pk_lo = -(1 << 30);
+    p.pk_hi = 1 << 30;
+    if (peer) {
+        p.pk_lo = peer->pk_lo; p.pk_hi = peer->pk_hi;
+        p.lo_koff = peer->lo_koff; p.hi_koff = peer->hi_koff;
+        p.u_lo = peer->u_lo; p.u_hi = peer->u_hi;
+        p.pflags = peer->flags; p.pflags_lo = peer->flags_lo; p.pflags_hi = peer->flags_hi;
+        p.epoch = peer->epoch;
+    }
     to_coef(*coeffs, p.c);
 
     const bool strict = (flags & SAFARA_FLAG_STRICT) != 0;
@@ -232,8 +249,11 @@ int launch(const double *u, const double *f, double *r, const safara_dims_t &d, 
     // aux fields are requested: then each face point also reads u and writes
     // naux strided values, too much for a handful of SMs, so every compute
     // CTA takes a share before its march
+    const long long face_pts =
+        (long long)(2 * d.nx + 2 * (d.ny - 2)) * (fk_hi - fk_lo) + 2LL * (d.nx - 2) * (d.ny - 2);
     p.nface_cta = (g_tune.face_ctas && !aux && fk_hi > fk_lo && p.units > 0 && ncta < max_ctas)
-                      ? (int)std::min<long long>(max_ctas - ncta, 32) : 0;
+                      ? (int)std::min<long long>({max_ctas - ncta, 32, (face_pts + 4095) / 4096})
+                      : 0;
 
 #ifdef SAFARA_TIMELINE
     {   // debug builds only: a static per-CTA timestamp buffer, dumped at exit
@@ -427,7 +447,8 @@ int safara_rhs(const double *u, const double *forcing, double *rhs, int nx, int 
 
 static int slab_launch(const double *u_slab, const double *forcing_slab, double *rhs_slab,
                        const safara_dims_t *dims, int k0, int nzl, const safara_coeffs_t *coeffs,
-                       int flags, int part, void *stream, double *aux, int naux, int ska) {
+                       int flags, int part, void *stream, double *aux, int naux, int ska,
+                       const PeerCfg *peer = nullptr) {
     if (!dims) return SAFARA_ERR_ARG;
     if (part < SAFARA_PART_ALL || part > SAFARA_PART_EDGE) return SAFARA_ERR_ARG;
     if (nzl < 2 || k0 < 0 || k0 + nzl > dims->nz) return SAFARA_ERR_SHAPE;
@@ -450,7 +471,79 @@ static int slab_launch(const double *u_slab, const double *forcing_slab, double 
         fk_lo = fk_hi = 0;
     }
     return launch(u_slab, forcing_slab, rhs_slab, *dims, nzu, nzl, k0, 2, ka0, kb0, ka1, kb1, fk_lo,
-                  fk_hi, coeffs, flags, (cudaStream_t)stream, aux, naux, ska);
+                  fk_hi, coeffs, flags, (cudaStream_t)stream, aux, naux, ska, peer);
+}
+
+int safara_rhs_peer(const double *u_slab, const double *forcing_slab, double *rhs_slab,
+                    const safara_dims_t *dims, int k0, int nzl, const safara_peer_t *peer,
+                    const safara_coeffs_t *coeffs, int flags, void *stream) {
+    if (!dims || !peer) return SAFARA_ERR_ARG;
+    const bool has_lo = k0 > 0, has_hi = k0 + nzl < dims->nz;
+    if ((peer->u_lo != nullptr) != has_lo || (peer->u_hi != nullptr) != has_hi)
+        return SAFARA_ERR_ARG;
+    // neighbours own >= 2 planes: [k0_lo, k0) and [k0_hi, ...)
+    if (has_lo && !(peer->k0_lo <= k0 - 2 && peer->k0_lo >= 0)) return SAFARA_ERR_ARG;
+    if (has_hi && peer->k0_hi != k0 + nzl) return SAFARA_ERR_ARG;
+    if (((uintptr_t)peer->u_lo | (uintptr_t)peer->u_hi) & 15u) return SAFARA_ERR_ALIGN;
+    if (peer->epoch) {
+        if (!peer->flags || (peer->flags_lo != nullptr) != has_lo ||
+            (peer->flags_hi != nullptr) != has_hi)
+            return SAFARA_ERR_ARG;
+        if (((uintptr_t)peer->flags | (uintptr_t)peer->flags_lo | (uintptr_t)peer->flags_hi) & 7u)
+            return SAFARA_ERR_ALIGN;
+    }
+    PeerCfg pc;
+    pc.pk_lo = has_lo ? k0 : -(1 << 30);
+    pc.pk_hi = has_hi ? k0 + nzl : 1 << 30;
+    pc.lo_koff = has_lo ? 2 - peer->k0_lo : 0;  // neighbour local plane = k - k0_lo + 2
+    pc.hi_koff = has_hi ? 2 - peer->k0_hi : 0;
+    pc.u_lo = peer->u_lo;
+    pc.u_hi = peer->u_hi;
+    pc.flags = reinterpret_cast<unsigned long long *>(peer->flags);
+    pc.flags_lo = reinterpret_cast<unsigned long long *>(peer->flags_lo);
+    pc.flags_hi = reinterpret_cast<unsigned long long *>(peer->flags_hi);
+    pc.epoch = peer->epoch;
+    return slab_launch(u_slab, forcing_slab, rhs_slab, dims, k0, nzl, coeffs, flags,
+                       SAFARA_PART_ALL, stream, nullptr, 0, 0, &pc);
+}
+
+int safara_ipc_get(const void *dptr, void *handle, int64_t *offset) {
+    if (!dptr || !handle || !offset) return SAFARA_ERR_ARG;
+    static PFN_cuMemGetAddressRange_v3020 range = nullptr;
+    if (!range) {
+        void *fn = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuMemGetAddressRange", &fn, cudaEnableDefault, &q) !=
+                cudaSuccess || !fn)
+            return SAFARA_ERR_CUDA;
+        range = (PFN_cuMemGetAddressRange_v3020)fn;
+    }
+    CUdeviceptr base = 0;
+    size_t size = 0;
+    if (range(&base, &size, (CUdeviceptr)dptr) != CUDA_SUCCESS) return SAFARA_ERR_CUDA;
+    cudaIpcMemHandle_t h;
+    if (cudaIpcGetMemHandle(&h, (void *)base) != cudaSuccess) return SAFARA_ERR_CUDA;
+    static_assert(sizeof(h) == SAFARA_IPC_HANDLE_BYTES, "IPC handle size");
+    std::memcpy(handle, &h, sizeof(h));
+    *offset = (int64_t)((CUdeviceptr)dptr - base);
+    return SAFARA_OK;
+}
+
+int safara_ipc_open(const void *handle, int64_t offset, void **dptr) {
+    if (!handle || !dptr || offset < 0) return SAFARA_ERR_ARG;
+    cudaIpcMemHandle_t h;
+    std::memcpy(&h, handle, sizeof(h));
+    void *base = nullptr;
+    if (cudaIpcOpenMemHandle(&base, h, cudaIpcMemLazyEnablePeerAccess) != cudaSuccess)
+        return SAFARA_ERR_CUDA;
+    *dptr = (char *)base + offset;
+    return SAFARA_OK;
+}
+
+int safara_ipc_close(void *dptr, int64_t offset) {
+    if (!dptr || offset < 0) return SAFARA_ERR_ARG;
+    return cudaIpcCloseMemHandle((char *)dptr - offset) == cudaSuccess ? SAFARA_OK
+                                                                        : SAFARA_ERR_CUDA;
 }
 
 int safara_rhs_slab(const double *u_slab, const double *forcing_slab, double *rhs_slab,

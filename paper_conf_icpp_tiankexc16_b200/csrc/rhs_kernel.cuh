@@ -177,6 +177,77 @@ __device__ __forceinline__ void prefetch_tmap(const CUtensorMap *map) {
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(map)) : "memory");
 }
 
+// ---- fused peer halo (include/safara.h safara_rhs_peer) ----
+__device__ __forceinline__ unsigned long long ld_acquire_sys(const unsigned long long *p) {
+    unsigned long long v;
+    asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_release_sys(unsigned long long *p, unsigned long long v) {
+    asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ unsigned long long global_ns() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+// Acquire flag word `word` of this rank >= epoch (bounded wait: after ~2 s
+// count a timeout and go on, so a broken peer can never hang the GPU).
+__device__ __forceinline__ void peer_wait(const Params &P, int word) {
+    const unsigned long long *f = P.pflags + word;
+    if (ld_acquire_sys(f) >= P.epoch) return;
+    const unsigned long long t0 = global_ns();
+    while (ld_acquire_sys(f) < P.epoch) {
+        __nanosleep(200);
+        if (global_ns() - t0 > 2000000000ull) {
+            atomicAdd(P.pflags + SAFARA_PEER_TIMEOUTS, 1ull);
+            atomicOr(P.pflags + SAFARA_PEER_TIMEOUTS + 1, 1ull << word);  // which wait
+            return;
+        }
+    }
+}
+// Own column (element offset colo = i + sy*j) of global plane kk, which lies
+// outside the local range [pk_lo, pk_hi): a neighbour's owned plane, read over
+// NVLink after acquiring its READY word.  These are the only values a slab
+// needs from its neighbours (the zeta window); 0 beyond the global grid.
+__device__ __forceinline__ void peer_col(double (&a)[5], const Params &P, int kk, int colo) {
+    const bool lo = kk < P.pk_lo;
+    const double *base = lo ? P.u_lo : P.u_hi;
+    if (base == nullptr || kk < 0 || kk >= P.nz) {
+#pragma unroll
+        for (int m = 0; m < 5; ++m) a[m] = 0.0;
+        return;
+    }
+    if (P.epoch) peer_wait(P, lo ? SAFARA_PEER_LO_READY : SAFARA_PEER_HI_READY);
+    const double *p = base + (colo + SK(u) * (kk + (lo ? P.lo_koff : P.hi_koff)));
+#pragma unroll
+    for (int m = 0; m < 5; ++m) a[m] = __ldcg(p + SM(u) * m);
+}
+// Every CTA: this rank's u of this epoch is final (stream order) -- tell the
+// neighbours.
+__device__ __forceinline__ void peer_publish(const Params &P) {
+    if (P.epoch == 0 || threadIdx.x != 0) return;
+    __threadfence_system();
+    if (P.pflags_lo) st_release_sys(P.pflags_lo + SAFARA_PEER_HI_READY, P.epoch);
+    if (P.pflags_hi) st_release_sys(P.pflags_hi + SAFARA_PEER_LO_READY, P.epoch);
+}
+// Every CTA at exit (its peer loads are complete): the last one tells the
+// neighbours we are done reading their u and waits until they are done with
+// ours, so the grid completes only when u may be overwritten.
+__device__ __forceinline__ void peer_arrive(const Params &P) {
+    if (P.epoch == 0) return;
+    __syncthreads();
+    if (threadIdx.x != 0) return;
+    __threadfence_system();
+    const unsigned long long old = atomicAdd(P.pflags + SAFARA_PEER_ARRIVED, 1ull);
+    if (old != (unsigned long long)gridDim.x - 1) return;
+    P.pflags[SAFARA_PEER_ARRIVED] = 0;  // next epoch's grid is stream-ordered after us
+    if (P.pflags_lo) st_release_sys(P.pflags_lo + SAFARA_PEER_HI_DONE, P.epoch);
+    if (P.pflags_hi) st_release_sys(P.pflags_hi + SAFARA_PEER_LO_DONE, P.epoch);
+    if (P.pflags_lo) peer_wait(P, SAFARA_PEER_LO_DONE);
+    if (P.pflags_hi) peer_wait(P, SAFARA_PEER_HI_DONE);
+}
+
 // NAS second difference  (a[p] - 2.0*a[c]) + a[q]; 2.0*a[c] is exact, so the
 // fused form rounds exactly like the two-step form.
 __device__ __forceinline__ double d2(double ap, double ac, double aq) {
@@ -484,6 +555,10 @@ __device__ __forceinline__ void issue_plane(const CUtensorMap *umap, const CUten
                                             const Params &P, double *su, uint64_t *full, int i0,
                                             int j0, int k, bool with_f, uint32_t seq) {
     const int slot = (int)(seq % STAGES);
+    if (k >= P.pk_hi) {  // f2: a neighbour's plane (own column read by peer_col)
+        mbar_arrive(&full[slot]);
+        return;
+    }
     const int kb = k - P.k0 + P.ukoff;
     const int kf = k - P.k0;
     const int jc = j0 - 2;
@@ -796,7 +871,15 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensor
 #endif
     // u(k+2) completes the zeta dissipation of plane k (production applies
     // it last, STRICT right after the zeta fluxes -- the NAS order)
-    load5(an, s2, g.uc);
+    if (k + 2 < P.pk_hi) {
+        load5(an, s2, g.uc);
+    } else {  // f2: plane k+2 belongs to the upper neighbour
+        unsigned lane;
+        asm("mov.u32 %0, %%laneid;" : "=r"(lane));
+        const int i = min(s_range[4] + (int)lane, P.nx - 1);
+        const int j = min(s_range[5] + (int)(threadIdx.x / TX), P.ny - 1);
+        peer_col(an, P, k + 2, i + P.sy * j);
+    }
     {
         double t_z[5];
         zeta_diss(t_z);
@@ -857,9 +940,11 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensor
     // Extra CTAs beyond the compute grid (on SMs the lockstep schedule leaves
     // idle) only copy the boundary faces.
     grid_dep_launch();
+    peer_publish(P);
     if ((int)blockIdx.x >= P.ncta) {
         grid_dep_wait();
         copy_faces<AUX>(P, (int)blockIdx.x - P.ncta, P.nface_cta);
+        peer_arrive(P);
 #ifdef SAFARA_TIMELINE
         if (threadIdx.x == 0 && P.dbg) {
             unsigned long long t_end;
@@ -984,22 +1069,34 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensor
             const int ic = min(i, P.nx - 1), jc = min(j, P.ny - 1);
             const int lk = ka - P.k0 + P.ukoff;  // local u plane of ka
             const double *uc0 = P.u + (idx_t)(ic + SY(u) * jc);
+            const int colo = ic + P.sy * jc;
+            if (ka - 1 < P.pk_lo) {
+                peer_col(g.a[0], P, ka - 1, colo);
+            } else {
 #pragma unroll
-            for (int m = 0; m < 5; ++m)
-                g.a[0][m] = lk - 1 >= 0 ? __ldg(uc0 + SM(u) * m + SK(u) * (lk - 1)) : 0.0;
+                for (int m = 0; m < 5; ++m)
+                    g.a[0][m] = lk - 1 >= 0 ? __ldg(uc0 + SM(u) * m + SK(u) * (lk - 1)) : 0.0;
+            }
             wait_plane(full, g.seq0);
             load5(g.a[1], su + (size_t)(g.seq0 % STAGES) * SLOT, g.uc);
             {
                 double am2[5];
+                if (ka - 2 < P.pk_lo) {
+                    peer_col(am2, P, ka - 2, colo);
+                } else {
 #pragma unroll
-                for (int m = 0; m < 5; ++m)
-                    am2[m] = lk - 2 >= 0 ? __ldg(uc0 + SM(u) * m + SK(u) * (lk - 2)) : 0.0;
+                    for (int m = 0; m < 5; ++m)
+                        am2[m] = lk - 2 >= 0 ? __ldg(uc0 + SM(u) * m + SK(u) * (lk - 2)) : 0.0;
+                }
                 zeta_partial(g.tp, am2, g.a[0], g.a[1], ka, P.nz, is_mid(ka, P.nz));
             }
             aux_of(g.a[0][0], g.a[0][1], g.a[0][2], g.a[0][3], g.ra[0], g.sa[0]);
             aux_of(g.a[1][0], g.a[1][1], g.a[1][2], g.a[1][3], g.ra[1], g.sa[1]);
             wait_plane(full, g.seq0 + 1);
-            load5(g.a[2], su + (size_t)((g.seq0 + 1) % STAGES) * SLOT, g.uc);
+            if (ka + 1 < P.pk_hi)
+                load5(g.a[2], su + (size_t)((g.seq0 + 1) % STAGES) * SLOT, g.uc);
+            else
+                peer_col(g.a[2], P, ka + 1, colo);
         }
 
         int k = ka;
@@ -1021,6 +1118,7 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensor
         if (tid == 0) s_range[0] = s_range[3];
         __syncthreads();
     }
+    peer_arrive(P);
 #ifdef SAFARA_TIMELINE
     if (tid == 0 && P.dbg) {
         unsigned long long t_end;

@@ -79,6 +79,18 @@ struct Params {
                            // local plane kl at i + sy*j + sm*c + ska*kl
     int naux;              // 6 (rho_i, us, vs, ws, square, qs) or 7 (+ SP speed)
     int ska;               // aux plane stride
+    // SURVEY §8(f) f2 (fused peer halo).  Global planes [pk_lo, pk_hi) are
+    // read from the local u buffer; a plane k < pk_lo comes from the lower
+    // neighbour's slab at u_lo + sk*(k + lo_koff), k >= pk_hi from the upper
+    // one at u_hi + sk*(k + hi_koff) (peer pointers over NVLink).  Single-GPU
+    // and ghost-slab launches: pk_lo = -2^30, pk_hi = 2^30, no peers.
+    int pk_lo, pk_hi;
+    int lo_koff, hi_koff;
+    const double *u_lo, *u_hi;
+    // Cross-GPU synchronisation (epoch > 0): pflags = this rank's flag words
+    // (SAFARA_PEER_* indices), pflags_lo / pflags_hi = the neighbours'.
+    unsigned long long *pflags, *pflags_lo, *pflags_hi;
+    unsigned long long epoch;
     unsigned long long *dbg;  // SAFARA_TIMELINE builds: per-CTA {start, end, smid}
     Coef c;
 };

@@ -11,6 +11,14 @@ The exchange uses torch.distributed P2P (NCCL over NVLink on GPUs, gloo on CPU
 for tests).  `rhs_sharded` overlaps it with the ghost-independent planes:
 PART_INTERIOR runs on the compute stream while the exchange is in flight,
 PART_EDGE after the exchange completes.
+
+SURVEY §8(f) f2, `rhs_fused`: no exchange at all.  The only values a slab
+needs from a neighbour are the own (i, j) columns of the two planes beyond its
+end (the zeta register window), so the kernel (safara_rhs_peer) loads them
+straight from the neighbours' u slabs over NVLink.  `PeerHalo` maps the
+neighbours' slabs and flag words into this process (CUDA IPC handles passed
+through the process group) and numbers the passes (epochs) that the kernel's
+release/acquire flags synchronise.
 """
 from __future__ import annotations
 
@@ -19,7 +27,7 @@ from dataclasses import dataclass
 import torch
 import torch.distributed as dist
 
-from ._abi import SAFARA_PART_EDGE, SAFARA_PART_INTERIOR
+from ._abi import SAFARA_PART_EDGE, SAFARA_PART_INTERIOR, SAFARA_PEER_WORDS, Peer
 
 GHOST = 2
 
@@ -106,4 +114,99 @@ def rhs_sharded(s: Slab, coeffs, comm_stream: torch.cuda.Stream | None = None,
     compute.wait_stream(comm)
     rhs_slab(s.u, s.forcing, s.rhs, s.nx, s.nz, s.k0, coeffs, part=SAFARA_PART_EDGE,
              strict=strict, stream=compute)
+    return s.rhs
+
+
+# ---- the halo fused into the pass --------------------------
+
+def neighbours(nz: int, p: int, rank: int) -> dict:
+    """Which neighbours rank ``rank`` reads and where their slabs start.
+
+    k0_lo / k0_hi: first global plane the lower / upper neighbour owns (None
+    at the grid ends).  Plane k of a neighbour sits at its local u plane
+    k - k0_nb + GHOST (the make_slab layout)."""
+    parts = partition(nz, p)
+    k0, nzl = parts[rank]
+    return {"k0": k0, "nzl": nzl,
+            "lo": rank - 1 if rank > 0 else None,
+            "hi": rank + 1 if rank < p - 1 else None,
+            "k0_lo": parts[rank - 1][0] if rank > 0 else None,
+            "k0_hi": k0 + nzl if rank < p - 1 else None}
+
+
+def peer_struct(nb: dict, u_lo: int | None, u_hi: int | None, flags: int | None,
+                flags_lo: int | None, flags_hi: int | None, epoch: int) -> Peer:
+    """safara_peer_t from raw device pointers (0/None = absent)."""
+    pr = Peer()
+    pr.u_lo = u_lo or None
+    pr.u_hi = u_hi or None
+    pr.k0_lo = nb["k0_lo"] if nb["k0_lo"] is not None else 0
+    pr.k0_hi = nb["k0_hi"] if nb["k0_hi"] is not None else 0
+    pr.flags = flags or None
+    pr.flags_lo = (flags_lo or None) if epoch else None
+    pr.flags_hi = (flags_hi or None) if epoch else None
+    pr.epoch = int(epoch)
+    return pr
+
+
+def new_flags(device) -> torch.Tensor:
+    """A rank's zeroed SAFARA_PEER_WORDS flag words."""
+    return torch.zeros(SAFARA_PEER_WORDS, dtype=torch.int64, device=device)
+
+
+class PeerHalo:
+    """Peer mapping of the neighbours' u slabs and flag words (one per rank).
+
+    Exports this rank's u slab and flags as CUDA IPC handles, gathers every
+    rank's through the process group (all_gather_object) and maps the two
+    neighbours'.  ``peer()`` returns the safara_peer_t of the next pass
+    (epoch + 1; ``sync=False`` -> epoch 0, inputs static)."""
+
+    def __init__(self, s: Slab, group=None):
+        from .rhs import ipc_get, ipc_open
+        self.slab = s
+        self.flags = new_flags(s.u.device)
+        self.nb = neighbours(s.nz, s.world, s.rank)
+        mine = (ipc_get(s.u), ipc_get(self.flags))
+        allx = [None] * s.world
+        dist.all_gather_object(allx, mine, group=group)
+        self._opened = []
+
+        def open_(r):
+            (hu, ou), (hf, of) = allx[r]
+            pu, pf = ipc_open(hu, ou), ipc_open(hf, of)
+            self._opened += [(pu, ou), (pf, of)]
+            return pu, pf
+
+        self.u_lo = self.f_lo = self.u_hi = self.f_hi = None
+        if self.nb["lo"] is not None:
+            self.u_lo, self.f_lo = open_(self.nb["lo"])
+        if self.nb["hi"] is not None:
+            self.u_hi, self.f_hi = open_(self.nb["hi"])
+        self.epoch = 0
+
+    def peer(self, sync: bool = True) -> Peer:
+        if sync:
+            self.epoch += 1
+        return peer_struct(self.nb, self.u_lo, self.u_hi, self.flags.data_ptr(), self.f_lo,
+                           self.f_hi, self.epoch if sync else 0)
+
+    def timeouts(self) -> int:
+        from ._abi import SAFARA_PEER_TIMEOUTS
+        return int(self.flags[SAFARA_PEER_TIMEOUTS].item())
+
+    def close(self):
+        from .rhs import ipc_close
+        for ptr, off in self._opened:
+            ipc_close(ptr, off)
+        self._opened = []
+
+
+def rhs_fused(s: Slab, halo: PeerHalo, coeffs, strict: bool = False, sync: bool = True,
+              stream=None) -> torch.Tensor:
+    """One distributed pass, halo fused into the kernel (one launch, no
+    exchange): f2."""
+    from .rhs import rhs_peer
+    rhs_peer(s.u, s.forcing, s.rhs, s.nx, s.nz, s.k0, halo.peer(sync), coeffs, strict=strict,
+             stream=stream)
     return s.rhs

@@ -13,8 +13,8 @@ import ctypes
 import numpy as np
 import torch
 
-from ._abi import (SAFARA_AUX_BT, SAFARA_AUX_SP, SAFARA_FLAG_STRICT, SAFARA_PART_ALL, Coeffs,
-                   Dims, Dims3, KernelInfo, check, lib)
+from ._abi import (SAFARA_AUX_BT, SAFARA_AUX_SP, SAFARA_FLAG_STRICT, SAFARA_IPC_HANDLE_BYTES,
+                   SAFARA_PART_ALL, Coeffs, Dims, Dims3, KernelInfo, Peer, check, lib)
 
 _initialised: set[int] = set()
 
@@ -117,6 +117,43 @@ def rhs_slab(u_slab: torch.Tensor, forcing_slab: torch.Tensor, out_slab: torch.T
                                 ctypes.byref(dims), int(k0), int(nzl), ctypes.byref(coeffs),
                                 flags, int(part), _stream_ptr(stream)), "safara_rhs_slab")
     return out_slab
+
+
+def rhs_peer(u_slab: torch.Tensor, forcing_slab: torch.Tensor, out_slab: torch.Tensor,
+             nx: int, nz: int, k0: int, peer: Peer, coeffs: Coeffs, strict: bool = False,
+             stream=None) -> torch.Tensor:
+    """f2: z-slab pass whose halo planes are read from the neighbours' u slabs
+    through the peer pointers in ``peer`` (safara_peer_t); one launch, no
+    exchange.  Slab tensors as in :func:`rhs_slab` (ghost planes unused)."""
+    for t, n in ((u_slab, "u_slab"), (forcing_slab, "forcing_slab"), (out_slab, "out_slab")):
+        _check_field(t, n)
+    nzl, _, ny, _ = forcing_slab.shape
+    dims = canonical_dims(nx, ny, nz)
+    flags = SAFARA_FLAG_STRICT if strict else 0
+    check(lib().safara_rhs_peer(u_slab.data_ptr(), forcing_slab.data_ptr(), out_slab.data_ptr(),
+                                ctypes.byref(dims), int(k0), int(nzl), ctypes.byref(peer),
+                                ctypes.byref(coeffs), flags, _stream_ptr(stream)),
+          "safara_rhs_peer")
+    return out_slab
+
+
+def ipc_get(t: torch.Tensor) -> tuple[bytes, int]:
+    """(handle bytes, offset) exporting the allocation that holds ``t``."""
+    h = ctypes.create_string_buffer(SAFARA_IPC_HANDLE_BYTES)
+    off = ctypes.c_int64()
+    check(lib().safara_ipc_get(t.data_ptr(), h, ctypes.byref(off)), "safara_ipc_get")
+    return h.raw, int(off.value)
+
+
+def ipc_open(handle: bytes, offset: int) -> int:
+    """Map another process's export on the current device; returns the pointer."""
+    p = ctypes.c_void_p()
+    check(lib().safara_ipc_open(handle, int(offset), ctypes.byref(p)), "safara_ipc_open")
+    return int(p.value)
+
+
+def ipc_close(ptr: int, offset: int) -> None:
+    check(lib().safara_ipc_close(ptr, int(offset)), "safara_ipc_close")
 
 
 def rhs_host(u_host: torch.Tensor, f_host: torch.Tensor, r_host: torch.Tensor,
