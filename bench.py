@@ -50,6 +50,10 @@ def parse():
                          "PAPER.md Fig. 8 loop (f4) on --seismic-n^3")
     ap.add_argument("--seismic-n", type=int, default=256)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--halo", default="peer", choices=["peer", "nccl"],
+                    help="N>1: peer = halo fused into the kernel (loads from the neighbours' "
+                         "slabs over NVLink, SURVEY f2); nccl = NCCL send/recv exchange "
+                         "overlapped with the interior planes (SURVEY §8(e))")
     ap.add_argument("--launch-events", action="store_true",
                     help="record an event after every launch (diagnostic; an event between "
                          "launches also serialises programmatic dependent launch)")

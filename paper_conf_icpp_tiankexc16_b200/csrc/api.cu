@@ -257,23 +257,31 @@ int launch(const double *u, const double *f, double *r, const safara_dims_t &d, 
 
 #ifdef SAFARA_TIMELINE
     {   // debug builds only: a static per-CTA timestamp buffer, dumped at exit
+        // the last 4 launches, ring-indexed by launch number; the dump lists
+        // them oldest first as "launch cta start end smid|cycles<<16"
         static unsigned long long *buf = nullptr;
         static int nct = 0;
+        static long long nl = 0;
         if (!buf) {
-            cudaMalloc(&buf, 3 * 1024 * sizeof(unsigned long long));
+            cudaMalloc(&buf, 4 * 3 * 1024 * sizeof(unsigned long long));
             std::atexit([] {
-                unsigned long long h[3 * 1024];
+                static unsigned long long h[4 * 3 * 1024];
                 cudaDeviceSynchronize();
                 cudaMemcpy(h, buf, sizeof(h), cudaMemcpyDeviceToHost);
                 FILE *f = std::fopen("gpurun_out/timeline.txt", "w");
                 if (f) {
-                    for (int c = 0; c < nct; ++c)
-                        std::fprintf(f, "%d %llu %llu %llu\n", c, h[3 * c], h[3 * c + 1], h[3 * c + 2]);
+                    for (long long l = std::max(0LL, nl - 4); l < nl; ++l) {
+                        const unsigned long long *b = h + 3 * 1024 * (l % 4);
+                        for (int c = 0; c < nct; ++c)
+                            std::fprintf(f, "%lld %d %llu %llu %llu\n", l, c, b[3 * c], b[3 * c + 1],
+                                         b[3 * c + 2]);
+                    }
                     std::fclose(f);
                 }
             });
         }
-        p.dbg = buf;
+        p.dbg = buf + 3 * 1024 * (nl % 4);
+        ++nl;
         nct = p.ncta + p.nface_cta;
     }
 #endif

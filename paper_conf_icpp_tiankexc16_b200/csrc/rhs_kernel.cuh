@@ -58,6 +58,12 @@
 #ifndef SAFARA_PROBE
 #define SAFARA_PROBE 0  // roofline probes: 1 memory only, 2 compute only (no TMA waits/refills, no stores), 3 no rhs stores
 #endif
+#ifndef SAFARA_PCHK_SPLIT
+#define SAFARA_PCHK_SPLIT 1  // main k loop without the f2 peer-plane check (0: one loop, checked)
+#endif
+#ifndef SAFARA_XREG
+#define SAFARA_XREG 1  // edge-tile xi case bits in a register (0: the smem table; A/B +-0.5 %)
+#endif
 #ifndef SAFARA_PDL
 #define SAFARA_PDL 0  // programmatic dependent launch (see launch_pdl; A/B on B200: no gain, profiles/ab_pdl_r01.txt)
 #endif
@@ -690,6 +696,9 @@ struct Seg {
     bool lane0, lane31;
     bool active, mid_x;
     int ycase;      // NAS dissipation case of row j: 0 mid, 1 j=1, 2 j=2, 3 j=ny-3, 4 j=ny-2
+#if SAFARA_XREG
+    int xo;         // edge tiles: i+-2 offsets and xi-dissipation case bits of this lane
+#endif
     uint32_t seq0;  // ring sequence number of the segment's first plane
     double a[3][5];      // u(:, i, j, k-1..k+1), rotating (see above)
     double ra[3], sa[3]; // rho_i / square of the same planes
@@ -716,7 +725,9 @@ __device__ __forceinline__ void zeta_partial(double (&tp)[5], const double (&am2
     }
 }
 
-template <int R, bool UD, bool AUX>
+// PCHK: plane k+2 may lie beyond the local slab (f2 peer halo; only the
+// last steps of a slab's march are instantiated with the check).
+template <int R, bool UD, bool AUX, bool PCHK>
 __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensorMap *umap,
                                          const CUtensorMap *fmap, int k) {
     constexpr int Q = R % 3, Z = (R + 1) % 3, PI = (R + 2) % 3;  // planes k-1, k, k+1
@@ -830,12 +841,22 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensor
                 // edge tile: absent i-2 / i+2 -> the zero-filled column beyond
                 unsigned lane;  // = tx
                 asm("mov.u32 %0, %%laneid;" : "=r"(lane));
+#if SAFARA_XREG
+                // per-lane case bits held in one register (no table loads)
+                const int xo = g.xo;
+                load5(pp, s, g.uc + (xo & 0xff));
+                load5(qq, s, g.uc - ((xo >> 8) & 0xff));
+                diss_terms_table(t, qq, q.u, wz, p.u, pp, (xo & (1 << 16)) ? -4.0 : 0.0,
+                                 (xo & (1 << 17)) ? 5.0 : 6.0, (xo & (1 << 18)) ? -4.0 : 0.0);
+                (void)lane;
+#else
                 const double *xc = smem_xcoef();
                 const int xo = reinterpret_cast<const int *>(xc + 3 * TX)[lane];
                 load5(pp, s, g.uc + (xo & 0xff));
                 load5(qq, s, g.uc - (xo >> 8));
                 diss_terms_table(t, qq, q.u, wz, p.u, pp, xc[lane], xc[TX + lane],
                                  xc[2 * TX + lane]);
+#endif
             }
         }
         flux_dir<1, false, UD>(acc, wz, vc, qsc, pc, p, q, C, 0);
@@ -871,7 +892,7 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensor
 #endif
     // u(k+2) completes the zeta dissipation of plane k (production applies
     // it last, STRICT right after the zeta fluxes -- the NAS order)
-    if (k + 2 < P.pk_hi) {
+    if (!PCHK || k + 2 < P.pk_hi) {
         load5(an, s2, g.uc);
     } else {  // f2: plane k+2 belongs to the upper neighbour
         unsigned lane;
@@ -1057,6 +1078,13 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensor
                 (i0 + tid == P.nx - 3 ? 3 : 2) | ((i0 + tid == 2 ? 3 : 2) << 8);
         }
         if (!g.mid_x) __syncthreads();  // the coefficient table is CTA-wide
+#if SAFARA_XREG
+        {
+            const Cases cs = cases_of(i0 + tx, P.nx);
+            g.xo = (i0 + tx == P.nx - 3 ? 3 : 2) | ((i0 + tx == 2 ? 3 : 2) << 8) |
+                   (cs.hm1 ? 1 << 16 : 0) | (cs.five ? 1 << 17 : 0) | (cs.hp1 ? 1 << 18 : 0);
+        }
+#endif
         g.ycase = is_mid(j, P.ny) ? 0 : j == 1 ? 1 : j == 2 ? 2 : j == P.ny - 3 ? 3 : 4;
         g.uc = (ty + 2) * UX + (tx + HX);  // centre in the u tile
         g.rptr = P.r + ((idx_t)i + SY(r) * j + SK(r) * (ka - P.k0));
@@ -1100,15 +1128,25 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensor
         }
 
         int k = ka;
+        // steps whose plane k+2 is local (all of them unless the slab's upper
+        // neighbour is a peer, f2) run without the peer check
+#if SAFARA_PCHK_SPLIT
 #pragma unroll 1
-        for (; k + 3 <= kb; k += 3) {
-            rhs_step<0, UD, AUX>(g, P, umap, fmap, k);
-            rhs_step<1, UD, AUX>(g, P, umap, fmap, k + 1);
-            rhs_step<2, UD, AUX>(g, P, umap, fmap, k + 2);
+        for (; k + 3 <= min(smem_kb(), P.pk_hi - 2); k += 3) {
+            rhs_step<0, UD, AUX, false>(g, P, umap, fmap, k);
+            rhs_step<1, UD, AUX, false>(g, P, umap, fmap, k + 1);
+            rhs_step<2, UD, AUX, false>(g, P, umap, fmap, k + 2);
+        }
+#endif
+#pragma unroll 1
+        for (; k + 3 <= smem_kb(); k += 3) {
+            rhs_step<0, UD, AUX, true>(g, P, umap, fmap, k);
+            rhs_step<1, UD, AUX, true>(g, P, umap, fmap, k + 1);
+            rhs_step<2, UD, AUX, true>(g, P, umap, fmap, k + 2);
         }
         if (k < kb) {
-            rhs_step<0, UD, AUX>(g, P, umap, fmap, k);
-            if (k + 1 < kb) rhs_step<1, UD, AUX>(g, P, umap, fmap, k + 1);
+            rhs_step<0, UD, AUX, true>(g, P, umap, fmap, k);
+            if (k + 1 < kb) rhs_step<1, UD, AUX, true>(g, P, umap, fmap, k + 1);
         }
         g.seq0 += (uint32_t)(s_range[2] - s_range[6] + 2);  // planes ka .. kb+1
         // Segment end: every warp has consumed every plane; planes kb, kb+1

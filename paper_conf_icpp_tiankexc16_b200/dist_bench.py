@@ -1,5 +1,9 @@
 """Multi-GPU arm of bench.py (torchrun, one rank per GPU, NCCL): BT class C
-split into z-slabs, one halo-exchanged compute_rhs pass per step.
+split into z-slabs, one compute_rhs pass per step.  --halo peer (default):
+the halo is fused into the kernel (safara_rhs_peer: one
+launch per rank per pass, neighbours' planes loaded over NVLink, epoch flags);
+--halo nccl: NCCL send/recv exchange overlapped with the interior planes
+(SURVEY §8(e)).
 
 Timing: barrier + synchronize on both sides of the K timed steps, CUDA events
 on each rank's compute stream, MAX over ranks (all_reduce).  value = all grid
@@ -19,14 +23,29 @@ def run(args):
     import nasgen
 
     from . import dist as sd
+    from bench import ClockSampler, measured_peaks
+
     from .rhs import coeffs_nas, init, kernel_info, launch_count, pack
 
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
     local = int(os.environ.get("LOCAL_RANK", str(rank)))
+    # SAFARA_SAME_GPU=1: every rank on GPU 0 with a gloo group -- a functional
+    # check of the whole multi-process path (IPC mapping, epochs, e2e, JSON)
+    # on a one-GPU box; its timings are time-sliced and mean nothing.
+    same_gpu = os.environ.get("SAFARA_SAME_GPU") == "1"
+    if world == 1:  # bench.py --dist without torchrun
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        os.environ.setdefault("MASTER_PORT", "29511")
+    if same_gpu:
+        local = 0
     torch.cuda.set_device(local)
-    dist.init_process_group("nccl", rank=rank, world_size=world,
-                            device_id=torch.device("cuda", local))
+    if same_gpu:
+        dist.init_process_group("gloo", rank=rank, world_size=world)
+    else:
+        dist.init_process_group("nccl", rank=rank, world_size=world,
+                                device_id=torch.device("cuda", local))
+    cdev = "cpu" if same_gpu else "cuda"  # collectives' tensors
     init(local)
     bench, cls = args.config.split("-")
     n, dt = nasgen.CLASSES[(bench, cls)]
@@ -36,12 +55,34 @@ def run(args):
     c = coeffs_nas(n, n, n, dt)
     comm = torch.cuda.Stream()
     compute = torch.cuda.current_stream()
+    halo = sd.PeerHalo(s) if args.halo == "peer" else None
 
     def step():
-        sd.rhs_sharded(s, c, comm_stream=comm, strict=args.strict)
+        if halo is not None:
+            sd.rhs_fused(s, halo, c, strict=args.strict, stream=compute)
+        else:
+            sd.rhs_sharded(s, c, comm_stream=comm, strict=args.strict)
 
+    w0, w1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    w0.record(compute)
     for _ in range(max(args.warmup, 3)):
         step()
+    w1.record(compute)
+    torch.cuda.synchronize()
+    # untimed soak so the clock sampler sees the loaded GPU; every rank runs
+    # the same number of passes (the peer halo pairs epochs across ranks)
+    wms = torch.tensor([w0.elapsed_time(w1) / max(args.warmup, 3)], device=cdev)
+    dist.all_reduce(wms, op=dist.ReduceOp.MAX)
+    nsoak = int(min(20000, args.soak_s * 1e3 / max(wms.item(), 1e-3)))
+    dist.barrier()
+    sampler = None
+    if rank == 0:
+        sampler = ClockSampler(local)
+        sampler.start()
+    for t in range(nsoak):
+        step()
+        if t % 50 == 49:
+            torch.cuda.synchronize()
     torch.cuda.synchronize()
     dist.barrier()
     l0 = launch_count()
@@ -52,9 +93,9 @@ def run(args):
     e1.record(compute)
     torch.cuda.synchronize()
     dist.barrier()
-    ms = torch.tensor([e0.elapsed_time(e1)], device="cuda")
+    ms = torch.tensor([e0.elapsed_time(e1)], device=cdev)
     dist.all_reduce(ms, op=dist.ReduceOp.MAX)
-    launches = torch.tensor([launch_count() - l0], device="cuda", dtype=torch.int64)
+    launches = torch.tensor([launch_count() - l0], device=cdev, dtype=torch.int64)
     dist.all_reduce(launches)
     ms_per_step = ms.item() / args.steps
     pts = n ** 3
@@ -77,24 +118,45 @@ def run(args):
     t1.record(compute)
     torch.cuda.synchronize()
     dist.barrier()
-    ems = torch.tensor([t0.elapsed_time(t1) / args.e2e_steps], device="cuda")
+    ems = torch.tensor([t0.elapsed_time(t1) / args.e2e_steps], device=cdev)
     dist.all_reduce(ems, op=dist.ReduceOp.MAX)
+    io = torch.tensor([(hu.numel() + hf.numel()) * 8, hr.numel() * 8,
+                       halo.timeouts() if halo is not None else 0], device=cdev,
+                      dtype=torch.int64)
+    dist.all_reduce(io)
+    clocks = ClockSampler.summarise(sampler.stop()) if sampler is not None else None
+    if halo is not None:
+        torch.cuda.synchronize()
+        dist.barrier()          # nobody unmaps a slab a neighbour may still read
+        halo.close()
 
     if rank == 0:
+        peak, peak_kind = measured_peaks()
+        achieved = 120 * pts / (ms_per_step * 1e-3) / 1e9
         line = {
             "metric": "rhs grid-points/s", "value": value, "unit": "Gpt/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_per_step,
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
             "data": "synthetic",
             "config": {"workload": nasgen.config_name(bench, cls), "grid": [n, n, n],
-                       "points": pts, "parallelism": f"z-slab x{world}, 2-plane NCCL halo",
+                       "points": pts,
+                       "parallelism": (f"z-slab x{world}, halo fused into the kernel (NVLink "
+                                       "peer loads, epoch flags)" if halo is not None else
+                                       f"z-slab x{world}, 2-plane NCCL send/recv halo"),
                        "variant": "strict" if args.strict else "production",
                        "l2": "per-rank slabs; inputs > L2 at C/1-2, no flush"},
-            "hbm_gbs": 120 * pts / (ms_per_step * 1e-3) / 1e9,
+            "hbm_gbs": achieved,
+            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak * world,
+                         "unit": "GB/s", "frac": achieved / (peak * world),
+                         "peak_kind": f"{peak_kind} per-GPU x {world}", "traffic": None,
+                         "bytes_per_point": 120, "kernel_ms": ms_per_step},
+            "clocks": clocks,
             "e2e": {"value": pts / (ems.item() * 1e-3) / 1e9, "unit": "Gpt/s",
-                    "h2d_bytes_per_step": int((hu.numel() + hf.numel()) * 8),
-                    "d2h_bytes_per_step": int(hr.numel() * 8), "note": "rank 0 slab bytes"},
+                    "h2d_bytes_per_step": int(io[0].item()),
+                    "d2h_bytes_per_step": int(io[1].item()),
+                    "note": "every rank copies its slab (u incl. ghosts, forcing) in and rhs out"},
             "gpu_launches": int(launches.item()),
+            "peer_wait_timeouts": int(io[2].item()),
             "kernel": kernel_info(args.strict),
         }
         print(json.dumps(line), flush=True)
