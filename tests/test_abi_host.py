@@ -106,3 +106,52 @@ def test_compute_without_init_fails_loudly(L):
     # No GPU here: the compute entry must return an error, never run on the CPU.
     rc = L.safara_rhs(1 << 20, 2 << 20, 3 << 20, 12, 12, 12, ctypes.byref(_abi.Coeffs()), None)
     assert rc < 0
+
+
+def test_peer_struct_layout_matches_header(tmp_path):
+    """safara_peer_t as the C compiler lays it out == the ctypes mirror."""
+    src = tmp_path / "peer.c"
+    src.write_text('#include <stddef.h>\n#include <stdio.h>\n#include "safara.h"\n'
+                   'int main(void){printf("%zu %zu %zu %zu %zu %zu %zu %zu %zu\\n",'
+                   'sizeof(safara_peer_t), offsetof(safara_peer_t,u_lo),'
+                   'offsetof(safara_peer_t,u_hi), offsetof(safara_peer_t,k0_lo),'
+                   'offsetof(safara_peer_t,k0_hi), offsetof(safara_peer_t,flags),'
+                   'offsetof(safara_peer_t,flags_lo), offsetof(safara_peer_t,flags_hi),'
+                   'offsetof(safara_peer_t,epoch));return 0;}\n')
+    exe = tmp_path / "peer"
+    inc = build.INCLUDE
+    subprocess.run(["gcc", "-I", inc, str(src), "-o", str(exe)], check=True)
+    got = [int(x) for x in subprocess.run([str(exe)], capture_output=True,
+                                          text=True).stdout.split()]
+    P = _abi.Peer
+    want = [ctypes.sizeof(P)] + [getattr(P, f).offset for f in
+                                  ("u_lo", "u_hi", "k0_lo", "k0_hi", "flags", "flags_lo",
+                                   "flags_hi", "epoch")]
+    assert got == want
+
+
+def test_peer_neighbours_and_struct():
+    from paper_conf_icpp_tiankexc16_b200 import dist as sd
+    nb = [sd.neighbours(162, 8, r) for r in range(8)]
+    assert nb[0]["lo"] is None and nb[0]["k0_hi"] == 21 and nb[7]["hi"] is None
+    for r in range(1, 8):
+        # the lower neighbour's slab ends where this one starts, and owns >= 2 planes
+        assert nb[r]["k0_lo"] == nb[r - 1]["k0"]
+        assert nb[r]["k0"] - nb[r]["k0_lo"] >= 2
+        assert nb[r - 1]["k0_hi"] == nb[r]["k0"]
+    pr = sd.peer_struct(nb[3], 0x1000, 0x2000, 0x3000, 0x4000, 0x5000, 0)
+    assert pr.u_lo == 0x1000 and pr.u_hi == 0x2000 and pr.flags_lo is None  # epoch 0: no flags
+    pr = sd.peer_struct(nb[0], None, 0x2000, 0x3000, None, 0x5000, 7)
+    assert pr.u_lo is None and pr.flags_hi == 0x5000 and pr.epoch == 7 and pr.k0_hi == 21
+
+
+def test_rhs_peer_rejects_bad_arguments_without_gpu(L):
+    """Argument checks run before any device work (no GPU needed)."""
+    d = sr.canonical_dims(12, 12, 12)
+    c = sr.coeffs_nas(12, 12, 12, 0.01)
+    pr = _abi.Peer()
+    # NULL peer struct / NULL dims
+    assert L.safara_rhs_peer(16, 16, 16, None, 0, 6, ctypes.byref(pr), ctypes.byref(c), 0,
+                             None) != 0
+    assert L.safara_rhs_peer(16, 16, 16, ctypes.byref(d), 0, 6, None, ctypes.byref(c), 0,
+                             None) != 0
