@@ -54,6 +54,13 @@ def parse():
                     help="N>1: peer = halo fused into the kernel (loads from the neighbours' "
                          "slabs over NVLink, SURVEY f2); nccl = NCCL send/recv exchange "
                          "overlapped with the interior planes (SURVEY §8(e))")
+    ap.add_argument("--graph", type=int, default=0, metavar="G",
+                    help="N=1: capture G passes into one CUDA graph and replay it K/G times "
+                         "(the per-launch gap becomes a graph-internal one)")
+    ap.add_argument("--slab-sim", type=int, default=0, metavar="P",
+                    help="one GPU: time the middle rank's fused-halo pass of a P-way "
+                         "z-split (neighbour slabs resident on the same GPU) next to the "
+                         "full-grid pass, and print the projected strong-scaling efficiency")
     ap.add_argument("--launch-events", action="store_true",
                     help="record an event after every launch (diagnostic; an event between "
                          "launches also serialises programmatic dependent launch)")
@@ -239,11 +246,31 @@ def run_single(args):
         da = sr.empty_aux(nx, ny, nz, sr.SAFARA_AUX_BT)
         bytes_per_point += 8 * sr.SAFARA_AUX_BT
 
-        def step():
-            sr.rhs_aux(du, df, dr, da, nx, c, strict=args.strict, stream=stream)
+        def step(st=None):
+            sr.rhs_aux(du, df, dr, da, nx, c, strict=args.strict, stream=st or stream)
     else:
-        def step():
-            sr.rhs(du, df, dr, nx, c, strict=args.strict, stream=stream)
+        def step(st=None):
+            sr.rhs(du, df, dr, nx, c, strict=args.strict, stream=st or stream)
+
+    graph, replays = None, 0
+    if args.graph > 0:
+        G = args.graph
+        args.steps = max(G, (args.steps // G) * G)
+        replays = args.steps // G
+        for _ in range(3):
+            step()
+        torch.cuda.synchronize()
+        graph = torch.cuda.CUDAGraph()
+        g0 = sr.launch_count()
+        with torch.cuda.graph(graph):
+            cs = torch.cuda.current_stream()
+            for _ in range(G):
+                step(cs)
+        per_graph_launches = sr.launch_count() - g0
+        torch.cuda.synchronize()
+
+        def step(st=None):  # noqa: F811 -- one replay = G passes
+            graph.replay()
 
     for _ in range(max(args.warmup, 3)):
         step()
@@ -262,18 +289,18 @@ def run_single(args):
     l0 = sr.launch_count()
     torch.cuda.synchronize()
     ev[0].record(stream)
-    for k in range(args.steps):
+    for k in range(replays if graph is not None else args.steps):
         step()
-        if args.launch_events:
+        if args.launch_events and graph is None:
             ev[k + 1].record(stream)
-    if not args.launch_events:
+    if not args.launch_events or graph is not None:
         ev[-1].record(stream)
     torch.cuda.synchronize()
-    launches = sr.launch_count() - l0
+    launches = sr.launch_count() - l0 + (per_graph_launches * replays if graph is not None else 0)
     total_ms = ev[0].elapsed_time(ev[-1])
     # one launch per step: the average launch duration is the step time
-    per = ([ev[k].elapsed_time(ev[k + 1]) for k in range(args.steps)] if args.launch_events
-           else [total_ms / args.steps])
+    per = ([ev[k].elapsed_time(ev[k + 1]) for k in range(args.steps)]
+           if args.launch_events and graph is None else [total_ms / args.steps])
     rows = sampler.stop()
     clocks = ClockSampler.summarise(rows)
 
@@ -312,7 +339,9 @@ def run_single(args):
         "config": {"workload": nasgen.config_name(bench, cls) if not args.grid else
                    f"{bench} compute_rhs {nx}x{ny}x{nz} fp64 (experiment grid)", "grid": [nx, ny, nz],
                    "points": pts, "variant": "strict" if args.strict else "production",
-                   "l2": "inputs 3x176 MB > 126 MB L2, no flush", "parallelism": "single"},
+                   "l2": "inputs 3x176 MB > 126 MB L2, no flush", "parallelism": "single",
+                   "launch": (f"CUDA graph of {args.graph} passes, replayed {replays}x"
+                              if graph is not None else "one stream launch per pass")},
         "hbm_gbs": achieved,
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "peak_kind": peak_kind, "traffic": traffic,
@@ -385,8 +414,78 @@ def run_seismic(args):
         "clocks": clocks, "gpu_launches": sr.launch_count() - l0}), flush=True)
 
 
+def run_slab_sim(args):
+    """Per-rank pass time of a P-way z-split, measured on one GPU: the middle
+    rank's safara_rhs_peer launch (its neighbours' slabs live on the same GPU,
+    epoch 0), K passes between two events, against the full-grid pass timed
+    the same way.  Projects T1 / (P * Tp); NVLink peer loads (2 x 2 own-column
+    planes per pass) and cross-GPU flag waits are not included."""
+    import torch
+
+    import nasgen
+    import paper_conf_icpp_tiankexc16_b200 as sr
+    from paper_conf_icpp_tiankexc16_b200 import dist as sd
+
+    torch.cuda.set_device(0)
+    sr.init(0)
+    bench, cls, n, dt = config_of(args)
+    inp = nasgen.make_class(bench, cls, seed=1)
+    c = sr.coeffs_nas(n, n, n, dt)
+    stream = torch.cuda.current_stream()
+
+    def timed(fn):
+        for _ in range(max(args.warmup, 3)):
+            fn()
+        torch.cuda.synchronize()
+        if args.graph > 0:
+            g = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(g):
+                for _ in range(args.graph):
+                    fn(torch.cuda.current_stream())
+            reps = max(1, args.steps // args.graph)
+            g.replay()
+            torch.cuda.synchronize()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            for _ in range(reps):
+                g.replay()
+            e1.record(stream)
+            torch.cuda.synchronize()
+            return e0.elapsed_time(e1) / (reps * args.graph)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(args.steps):
+            fn()
+        e1.record(stream)
+        torch.cuda.synchronize()
+        return e0.elapsed_time(e1) / args.steps
+
+    du, df = sr.pack(inp.u), sr.pack(inp.forcing)
+    dr = torch.empty_like(du)
+    t1 = timed(lambda st=None: sr.rhs(du, df, dr, n, c, stream=st or stream))
+    del du, df, dr
+    p = args.slab_sim
+    ug, fg = sr.pack(inp.u, device="cpu"), sr.pack(inp.forcing, device="cpu")
+    r = p // 2
+    nb = sd.neighbours(n, p, r)
+    slabs = {q: sd.make_slab(ug, fg, n, q, p, device="cuda") for q in (nb["lo"], r, nb["hi"])
+             if q is not None}
+    s = slabs[r]
+    pr = sd.peer_struct(nb, slabs[nb["lo"]].u.data_ptr() if nb["lo"] is not None else None,
+                        slabs[nb["hi"]].u.data_ptr() if nb["hi"] is not None else None,
+                        None, None, None, 0)
+    tp = timed(lambda st=None: sr.rhs_peer(s.u, s.forcing, s.rhs, n, n, s.k0, pr, c,
+                                           stream=st or stream))
+    print(json.dumps({"slab_sim": p, "rank": r, "planes": s.nzl, "config": f"{bench}-{cls}",
+                      "t1_ms": t1, "tp_ms": tp, "projected_efficiency": t1 / (p * tp),
+                      "steps": args.steps, "graph": args.graph}), flush=True)
+
+
 def main():
     args = parse()
+    if args.slab_sim:
+        run_slab_sim(args)
+        return
     if args.workload == "seismic_dz" and args.impl != "reference":
         run_seismic(args)
         return

@@ -175,6 +175,12 @@ int safara_rhs_slab(const double *u_slab, const double *forcing_slab,
 #define SAFARA_PEER_ARRIVED  4  /* own grid's CTA arrival counter           */
 #define SAFARA_PEER_TIMEOUTS 5  /* waits that gave up (should stay 0)       */
 #define SAFARA_PEER_TIMEOUT_WORDS 6  /* bit w set: a wait on word w gave up */
+#define SAFARA_PEER_EPOCH_WORD 7  /* the device epoch counter (EPOCH_AUTO)  */
+/* epoch = SAFARA_PEER_EPOCH_AUTO: the pass's epoch is flags[EPOCH_WORD] + 1,
+ * read on the device and advanced by the pass itself, so a captured CUDA
+ * graph of passes replays with fresh epochs (every rank must run the same
+ * number of passes, as with explicit epochs).                              */
+#define SAFARA_PEER_EPOCH_AUTO 0xffffffffffffffffull
 #define SAFARA_PEER_WORDS    8
 typedef struct {
     const double *u_lo, *u_hi;      /* neighbours' u slabs (peer pointers)   */

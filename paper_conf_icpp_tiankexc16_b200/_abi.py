@@ -59,6 +59,8 @@ class Peer(ctypes.Structure):
 SAFARA_PEER_WORDS = 8
 SAFARA_PEER_LO_READY, SAFARA_PEER_HI_READY, SAFARA_PEER_LO_DONE, SAFARA_PEER_HI_DONE = 0, 1, 2, 3
 SAFARA_PEER_ARRIVED, SAFARA_PEER_TIMEOUTS = 4, 5
+SAFARA_PEER_TIMEOUT_WORDS, SAFARA_PEER_EPOCH_WORD = 6, 7
+SAFARA_PEER_EPOCH_AUTO = 0xFFFFFFFFFFFFFFFF
 SAFARA_IPC_HANDLE_BYTES = 64
 
 _lock = threading.Lock()

@@ -49,11 +49,12 @@ DeviceState g_dev[kMaxDevices];
 // chunk-major work order (0 = whole column).  SAFARA_SCHED: 0 = balanced
 // contiguous ranges, 1 = lockstep (column tile, k-part) per CTA.
 struct Tune {
-    int l2promo = 0;
+    int l2promo = 3;  // 256 B (A/B: +0.3-0.4 % over none, profiles/ab_knobs_r01.txt)
     int chunk = 0;
     int sched = 1;  // 0 = balanced contiguous ranges, 1 = lockstep (column, k-part)
     int interleave = 1;  // lockstep CTA order: 1 = tile-major across CTAs, 0 = part-major
     int face_ctas = 1;   // boundary faces on the idle SMs' extra CTAs (else by compute CTAs)
+    int min_planes = MIN_PLANES_PER_CTA;  // shortest k-run a CTA is given
 } g_tune;
 
 int env_int(const char *name, int dflt) {
@@ -225,7 +226,7 @@ int launch(const double *u, const double *f, double *r, const safara_dims_t &d, 
     const long long max_ctas = (long long)std::max(per_sm, 1) * st.sms;
     long long ncta;
     long long parts = p.ncol > 0 ? max_ctas / p.ncol : 0;
-    parts = std::min<long long>(parts, std::max(1, p.nplanes / MIN_PLANES_PER_CTA));
+    parts = std::min<long long>(parts, std::max(1, p.nplanes / g_tune.min_planes));
     // Lockstep only when it keeps >= 90% of the CTA slots busy (e.g. class C:
     // 70 column tiles x 2 parts = 140 of 148); otherwise balanced ranges.
     const bool lockstep = g_tune.sched == 1 && parts >= 1 && p.nplanes > 0 &&
@@ -237,7 +238,7 @@ int launch(const double *u, const double *f, double *r, const safara_dims_t &d, 
         ncta = p.ncol * parts;
         p.parts = g_tune.interleave ? (int)parts : 0;
     } else {
-        ncta = (p.units + MIN_PLANES_PER_CTA - 1) / MIN_PLANES_PER_CTA;
+        ncta = (p.units + g_tune.min_planes - 1) / g_tune.min_planes;
         ncta = std::min(ncta, max_ctas);
     }
     if (ncta < 1) {
@@ -382,6 +383,7 @@ int safara_rhs_init(int device) {
     g_tune.sched = env_int("SAFARA_SCHED", g_tune.sched);
     g_tune.interleave = env_int("SAFARA_INTERLEAVE", g_tune.interleave);
     g_tune.face_ctas = env_int("SAFARA_FACE_CTAS", g_tune.face_ctas);
+    g_tune.min_planes = std::max(1, env_int("SAFARA_MIN_PLANES", g_tune.min_planes));
     int major = 0, minor = 0, sms = 0;
     if (cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, device) ||
         cudaDeviceGetAttribute(&minor, cudaDevAttrComputeCapabilityMinor, device) ||

@@ -58,6 +58,9 @@
 #ifndef SAFARA_PROBE
 #define SAFARA_PROBE 0  // roofline probes: 1 memory only, 2 compute only (no TMA waits/refills, no stores), 3 no rhs stores
 #endif
+#ifndef SAFARA_KBM_SMEM
+#define SAFARA_KBM_SMEM 1  // unchecked-march bound read from shared memory each iteration
+#endif
 #ifndef SAFARA_PCHK_SPLIT
 #define SAFARA_PCHK_SPLIT 1  // main k loop without the f2 peer-plane check (0: one loop, checked)
 #endif
@@ -179,6 +182,12 @@ __device__ __forceinline__ void grid_dep_wait() {
 #endif
 }
 
+__device__ __forceinline__ int reread(const int &x) {
+    int r;
+    asm volatile("mov.b32 %0, %1;" : "=r"(r) : "r"(x));
+    return r;
+}
+
 __device__ __forceinline__ void prefetch_tmap(const CUtensorMap *map) {
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(map)) : "memory");
 }
@@ -197,17 +206,30 @@ __device__ __forceinline__ unsigned long long global_ns() {
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
     return t;
 }
+// The pass's epoch: P.epoch, or with SAFARA_PEER_EPOCH_AUTO this rank's
+// device counter + 1 (read by every CTA at its start, advanced by the last
+// CTA at its end), so a CUDA graph of passes replays with fresh epochs.
+__shared__ unsigned long long s_epoch;
+__device__ __forceinline__ unsigned long long peer_epoch() { return s_epoch; }
+__device__ __forceinline__ void peer_epoch_init(const Params &P) {
+    if (threadIdx.x == 0)
+        s_epoch = P.epoch == SAFARA_PEER_EPOCH_AUTO
+                      ? *(volatile unsigned long long *)(P.pflags + SAFARA_PEER_EPOCH_WORD) + 1
+                      : P.epoch;
+}
+
 // Acquire flag word `word` of this rank >= epoch (bounded wait: after ~2 s
 // count a timeout and go on, so a broken peer can never hang the GPU).
 __device__ __forceinline__ void peer_wait(const Params &P, int word) {
+    const unsigned long long e = peer_epoch();
     const unsigned long long *f = P.pflags + word;
-    if (ld_acquire_sys(f) >= P.epoch) return;
+    if (ld_acquire_sys(f) >= e) return;
     const unsigned long long t0 = global_ns();
-    while (ld_acquire_sys(f) < P.epoch) {
+    while (ld_acquire_sys(f) < e) {
         __nanosleep(200);
         if (global_ns() - t0 > 2000000000ull) {
             atomicAdd(P.pflags + SAFARA_PEER_TIMEOUTS, 1ull);
-            atomicOr(P.pflags + SAFARA_PEER_TIMEOUTS + 1, 1ull << word);  // which wait
+            atomicOr(P.pflags + SAFARA_PEER_TIMEOUT_WORDS, 1ull << word);  // which wait
             return;
         }
     }
@@ -233,9 +255,10 @@ __device__ __forceinline__ void peer_col(double (&a)[5], const Params &P, int kk
 // neighbours.
 __device__ __forceinline__ void peer_publish(const Params &P) {
     if (P.epoch == 0 || threadIdx.x != 0) return;
+    const unsigned long long e = peer_epoch();
     __threadfence_system();
-    if (P.pflags_lo) st_release_sys(P.pflags_lo + SAFARA_PEER_HI_READY, P.epoch);
-    if (P.pflags_hi) st_release_sys(P.pflags_hi + SAFARA_PEER_LO_READY, P.epoch);
+    if (P.pflags_lo) st_release_sys(P.pflags_lo + SAFARA_PEER_HI_READY, e);
+    if (P.pflags_hi) st_release_sys(P.pflags_hi + SAFARA_PEER_LO_READY, e);
 }
 // Every CTA at exit (its peer loads are complete): the last one tells the
 // neighbours we are done reading their u and waits until they are done with
@@ -244,12 +267,14 @@ __device__ __forceinline__ void peer_arrive(const Params &P) {
     if (P.epoch == 0) return;
     __syncthreads();
     if (threadIdx.x != 0) return;
+    const unsigned long long e = peer_epoch();
     __threadfence_system();
     const unsigned long long old = atomicAdd(P.pflags + SAFARA_PEER_ARRIVED, 1ull);
     if (old != (unsigned long long)gridDim.x - 1) return;
     P.pflags[SAFARA_PEER_ARRIVED] = 0;  // next epoch's grid is stream-ordered after us
-    if (P.pflags_lo) st_release_sys(P.pflags_lo + SAFARA_PEER_HI_DONE, P.epoch);
-    if (P.pflags_hi) st_release_sys(P.pflags_hi + SAFARA_PEER_LO_DONE, P.epoch);
+    if (P.epoch == SAFARA_PEER_EPOCH_AUTO) P.pflags[SAFARA_PEER_EPOCH_WORD] = e;
+    if (P.pflags_lo) st_release_sys(P.pflags_lo + SAFARA_PEER_HI_DONE, e);
+    if (P.pflags_hi) st_release_sys(P.pflags_hi + SAFARA_PEER_LO_DONE, e);
     if (P.pflags_lo) peer_wait(P, SAFARA_PEER_LO_DONE);
     if (P.pflags_hi) peer_wait(P, SAFARA_PEER_HI_DONE);
 }
@@ -685,7 +710,8 @@ __device__ __forceinline__ double *smem_xcoef() {
 // This CTA's unit range [ub, ue) and the current segment's end plane kb
 // live in shared memory across the k march (CTA-uniform; keeps registers free
 // for the unrolled window).
-__shared__ int s_range[7];  // ub, ue, segment kb, next segment's ub, tile i0, j0, segment ka
+__shared__ int s_range[8];  // ub, ue, segment kb, next segment's ub, tile i0, j0, segment ka,
+                            // end of the unchecked k march (min(kb, pk_hi - 2))
 __device__ __forceinline__ int smem_kb() { return *(volatile int *)&s_range[2]; }
 
 struct Seg {
@@ -961,7 +987,11 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensor
     // Extra CTAs beyond the compute grid (on SMs the lockstep schedule leaves
     // idle) only copy the boundary faces.
     grid_dep_launch();
-    peer_publish(P);
+    if (P.epoch) {
+        peer_epoch_init(P);
+        __syncthreads();
+        peer_publish(P);
+    }
     if ((int)blockIdx.x >= P.ncta) {
         grid_dep_wait();
         copy_faces<AUX>(P, (int)blockIdx.x - P.ncta, P.nface_cta);
@@ -1050,11 +1080,15 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensor
             s_range[4] = i0;
             s_range[5] = j0;
             s_range[6] = g.ka;
+            s_range[7] = min(g.kb, P.pk_hi - 2);
         }
         const int ka = g.ka, kb = g.kb;
 
         const int i = i0 + tx, j = j0 + ty;
-        g.active = (i <= P.nx - 2) && (j <= P.ny - 2);
+        // extents re-read per segment (volatile: not hoisted into registers
+        // live across the march)
+        const int nx_s = reread(P.nx), ny_s = reread(P.ny);
+        g.active = (i <= nx_s - 2) && (j <= ny_s - 2);
         const int nload = kb - ka + 2;  // ring planes ka .. kb+1
 
         if (tid == 0 && !first) {
@@ -1085,7 +1119,7 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensor
                    (cs.hm1 ? 1 << 16 : 0) | (cs.five ? 1 << 17 : 0) | (cs.hp1 ? 1 << 18 : 0);
         }
 #endif
-        g.ycase = is_mid(j, P.ny) ? 0 : j == 1 ? 1 : j == 2 ? 2 : j == P.ny - 3 ? 3 : 4;
+        g.ycase = is_mid(j, ny_s) ? 0 : j == 1 ? 1 : j == 2 ? 2 : j == ny_s - 3 ? 3 : 4;
         g.uc = (ty + 2) * UX + (tx + HX);  // centre in the u tile
         g.rptr = P.r + ((idx_t)i + SY(r) * j + SK(r) * (ka - P.k0));
 
@@ -1094,7 +1128,7 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensor
         // the TMA ring.  Lanes outside the grid read the nearest in-grid
         // column (valid memory; they store nothing and feed no active lane).
         {
-            const int ic = min(i, P.nx - 1), jc = min(j, P.ny - 1);
+            const int ic = min(i, nx_s - 1), jc = min(j, ny_s - 1);
             const int lk = ka - P.k0 + P.ukoff;  // local u plane of ka
             const double *uc0 = P.u + (idx_t)(ic + SY(u) * jc);
             const int colo = ic + P.sy * jc;
@@ -1132,7 +1166,11 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensor
         // neighbour is a peer, f2) run without the peer check
 #if SAFARA_PCHK_SPLIT
 #pragma unroll 1
+#if SAFARA_KBM_SMEM
+        for (; k + 3 <= *(volatile int *)&s_range[7]; k += 3) {
+#else
         for (; k + 3 <= min(smem_kb(), P.pk_hi - 2); k += 3) {
+#endif
             rhs_step<0, UD, AUX, false>(g, P, umap, fmap, k);
             rhs_step<1, UD, AUX, false>(g, P, umap, fmap, k + 1);
             rhs_step<2, UD, AUX, false>(g, P, umap, fmap, k + 2);

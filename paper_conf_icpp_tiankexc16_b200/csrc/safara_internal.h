@@ -40,7 +40,7 @@ static_assert(STAGES * (8 + 4) <= XCOEF_OFF * 8, "mbarriers + release counters f
 // after the mbarriers: the edge-tile xi table, 3 coefficient rows (double)
 // and one row of packed i+-2 offsets (int)
 constexpr size_t SMEM_BYTES = (size_t)STAGES * SLOT * 8 + (XCOEF_OFF + 3 * TX + TX / 2) * 8;
-constexpr int MIN_PLANES_PER_CTA = 4;
+constexpr int MIN_PLANES_PER_CTA = 2;  // small slabs: more k-parts win (SP-B/8: 16.4 -> 12.5 us, profiles/slab_sim_r01.txt)
 
 // Device-side coefficients: safara_coeffs_t plus the constant products that
 // the NAS text evaluates left to right (xxcon2*con43 -> one double).
@@ -90,7 +90,7 @@ struct Params {
     // Cross-GPU synchronisation (epoch > 0): pflags = this rank's flag words
     // (SAFARA_PEER_* indices), pflags_lo / pflags_hi = the neighbours'.
     unsigned long long *pflags, *pflags_lo, *pflags_hi;
-    unsigned long long epoch;
+    unsigned long long epoch;  // 0: none; SAFARA_PEER_EPOCH_AUTO: device counter
     unsigned long long *dbg;  // SAFARA_TIMELINE builds: per-CTA {start, end, smid}
     Coef c;
 };

@@ -27,7 +27,8 @@ from dataclasses import dataclass
 import torch
 import torch.distributed as dist
 
-from ._abi import SAFARA_PART_EDGE, SAFARA_PART_INTERIOR, SAFARA_PEER_WORDS, Peer
+from ._abi import (SAFARA_PART_EDGE, SAFARA_PART_INTERIOR, SAFARA_PEER_EPOCH_AUTO,
+                   SAFARA_PEER_WORDS, Peer)
 
 GHOST = 2
 
@@ -185,7 +186,12 @@ class PeerHalo:
             self.u_hi, self.f_hi = open_(self.nb["hi"])
         self.epoch = 0
 
-    def peer(self, sync: bool = True) -> Peer:
+    def peer(self, sync: bool = True, auto: bool = False) -> Peer:
+        """safara_peer_t of the next pass.  auto: the epoch is counted on the
+        device (SAFARA_PEER_EPOCH_AUTO), for passes captured in a CUDA graph."""
+        if auto:
+            return peer_struct(self.nb, self.u_lo, self.u_hi, self.flags.data_ptr(), self.f_lo,
+                               self.f_hi, SAFARA_PEER_EPOCH_AUTO)
         if sync:
             self.epoch += 1
         return peer_struct(self.nb, self.u_lo, self.u_hi, self.flags.data_ptr(), self.f_lo,
@@ -203,10 +209,11 @@ class PeerHalo:
 
 
 def rhs_fused(s: Slab, halo: PeerHalo, coeffs, strict: bool = False, sync: bool = True,
-              stream=None) -> torch.Tensor:
+              stream=None, auto: bool = False) -> torch.Tensor:
     """One distributed pass, halo fused into the kernel (one launch, no
-    exchange): f2."""
+    exchange): f2.  Do not mix host-numbered (sync) and device-numbered
+    (auto) epochs on one PeerHalo."""
     from .rhs import rhs_peer
-    rhs_peer(s.u, s.forcing, s.rhs, s.nx, s.nz, s.k0, halo.peer(sync), coeffs, strict=strict,
-             stream=stream)
+    rhs_peer(s.u, s.forcing, s.rhs, s.nx, s.nz, s.k0, halo.peer(sync, auto), coeffs,
+             strict=strict, stream=stream)
     return s.rhs

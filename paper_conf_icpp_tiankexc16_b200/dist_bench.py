@@ -57,21 +57,46 @@ def run(args):
     compute = torch.cuda.current_stream()
     halo = sd.PeerHalo(s) if args.halo == "peer" else None
 
-    def step():
+    use_graph = args.graph > 0 and halo is not None
+
+    def step(st=None):
         if halo is not None:
-            sd.rhs_fused(s, halo, c, strict=args.strict, stream=compute)
+            # graph mode: device-counted epochs (the same struct replays)
+            sd.rhs_fused(s, halo, c, strict=args.strict, stream=st or compute, auto=use_graph)
         else:
             sd.rhs_sharded(s, c, comm_stream=comm, strict=args.strict)
 
+    if use_graph:
+        # G passes per CUDA graph (one launch gap per G passes); every rank
+        # captures and replays the same count, epochs advance on the device
+        for _ in range(3):
+            step()
+        torch.cuda.synchronize()
+        graph = torch.cuda.CUDAGraph()
+        g0 = launch_count()
+        with torch.cuda.graph(graph):
+            for _ in range(args.graph):
+                step(torch.cuda.current_stream())
+        per_graph = launch_count() - g0
+        G = args.graph
+        args.steps = max(G, (args.steps // G) * G)
+        torch.cuda.synchronize()
+        dist.barrier()
+        eager_step = step
+
+        def step(st=None):  # noqa: F811 -- one replay = G passes
+            graph.replay()
+
     w0, w1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     w0.record(compute)
-    for _ in range(max(args.warmup, 3)):
+    nstep = (lambda k: max(1, k // args.graph)) if use_graph else (lambda k: k)
+    for _ in range(nstep(max(args.warmup, 3))):
         step()
     w1.record(compute)
     torch.cuda.synchronize()
     # untimed soak so the clock sampler sees the loaded GPU; every rank runs
     # the same number of passes (the peer halo pairs epochs across ranks)
-    wms = torch.tensor([w0.elapsed_time(w1) / max(args.warmup, 3)], device=cdev)
+    wms = torch.tensor([w0.elapsed_time(w1) / nstep(max(args.warmup, 3))], device=cdev)
     dist.all_reduce(wms, op=dist.ReduceOp.MAX)
     nsoak = int(min(20000, args.soak_s * 1e3 / max(wms.item(), 1e-3)))
     dist.barrier()
@@ -88,14 +113,15 @@ def run(args):
     l0 = launch_count()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     e0.record(compute)
-    for _ in range(args.steps):
+    for _ in range(nstep(args.steps)):
         step()
     e1.record(compute)
     torch.cuda.synchronize()
     dist.barrier()
     ms = torch.tensor([e0.elapsed_time(e1)], device=cdev)
     dist.all_reduce(ms, op=dist.ReduceOp.MAX)
-    launches = torch.tensor([launch_count() - l0], device=cdev, dtype=torch.int64)
+    launches = torch.tensor([launch_count() - l0 + (per_graph * nstep(args.steps) if use_graph
+                                                    else 0)], device=cdev, dtype=torch.int64)
     dist.all_reduce(launches)
     ms_per_step = ms.item() / args.steps
     pts = n ** 3
@@ -113,7 +139,7 @@ def run(args):
     for _ in range(args.e2e_steps):
         s.u.copy_(hu, non_blocking=True)
         s.forcing.copy_(hf, non_blocking=True)
-        step()
+        (eager_step if use_graph else step)()
         hr.copy_(s.rhs, non_blocking=True)
     t1.record(compute)
     torch.cuda.synchronize()
@@ -141,7 +167,9 @@ def run(args):
             "config": {"workload": nasgen.config_name(bench, cls), "grid": [n, n, n],
                        "points": pts,
                        "parallelism": (f"z-slab x{world}, halo fused into the kernel (NVLink "
-                                       "peer loads, epoch flags)" if halo is not None else
+                                       "peer loads, epoch flags)" + (
+                                           f", CUDA graph of {args.graph} passes" if use_graph
+                                           else "") if halo is not None else
                                        f"z-slab x{world}, 2-plane NCCL send/recv halo"),
                        "variant": "strict" if args.strict else "production",
                        "l2": "per-rank slabs; inputs > L2 at C/1-2, no flush"},

@@ -206,6 +206,50 @@ def test_peer_epochs_concurrent(shape, p):
     _in_child(_epochs_body, shape, p)
 
 
+def _auto_graph_body(shape, p):
+    """SAFARA_PEER_EPOCH_AUTO: each rank captures 3 passes into its own CUDA
+    graph (the same peer struct in every node); the graphs replay
+    concurrently, twice, and the device epoch counter advances to 6."""
+    from paper_conf_icpp_tiankexc16_b200._abi import SAFARA_PEER_EPOCH_AUTO, SAFARA_PEER_EPOCH_WORD
+    nz, ny, nx = shape
+    inp = nasgen.make_inputs(nx, ny, nz, seed=8, B=1e-2, dt=0.002)
+    o = oracle.compute_rhs(inp.u, inp.forcing, dt=inp.dt, threads=8)
+    slabs = _slabs(inp, p)
+    flags = [sd.new_flags("cuda") for _ in range(p)]
+    streams = [torch.cuda.Stream() for _ in range(p)]
+    peers = _peers(slabs, flags, SAFARA_PEER_EPOCH_AUTO)
+    c = _c(inp)
+    torch.cuda._sleep(1000)
+    torch.cuda.synchronize()
+    graphs = []
+    for r, (s, pr) in enumerate(zip(slabs, peers)):
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, stream=streams[r]):
+            for _ in range(3):
+                sr.rhs_peer(s.u, s.forcing, s.rhs, nx, nz, s.k0, pr, c, strict=True,
+                            stream=streams[r])
+        graphs.append(g)
+    torch.cuda.synchronize()
+    for rep in range(2):
+        for s in slabs:
+            s.rhs.fill_(float("nan"))
+        torch.cuda.synchronize()
+        for r, g in enumerate(graphs):
+            with torch.cuda.stream(streams[r]):
+                g.replay()
+        torch.cuda.synchronize()
+        assert np.array_equal(_gather(slabs, nx), o), f"replay {rep}"
+    for f in flags:
+        f = f.cpu().tolist()
+        assert f[SAFARA_PEER_TIMEOUTS] == 0 and f[SAFARA_PEER_ARRIVED] == 0, f
+        assert f[SAFARA_PEER_EPOCH_WORD] == 6, f
+
+
+@pytest.mark.parametrize("shape,p", [((24, 34, 30), 2), ((20, 14, 40), 3)])
+def test_peer_auto_epoch_graphs(shape, p):
+    _in_child(_auto_graph_body, shape, p)
+
+
 def _waits_body():
     nz, ny, nx = 30, 34, 24
     p, mid = 3, 1

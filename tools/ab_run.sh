@@ -1,6 +1,7 @@
 cd $GRAFT_REPO_ROOT
-ncu --metrics gpu__time_duration.sum --clock-control none -c 30 --csv --log-file gpurun_out/launches.csv python bench.py --steps 10 --warmup 3 --no-cpu-baseline --e2e-steps 1 --soak-s 0 > gpurun_out/ncu_bench.log 2>&1
-ncu --set full --clock-control none --import-source on -k regex:rhs_kernel -s 5 -c 1 -o gpurun_out/prof -f python bench.py --steps 3 --warmup 3 --no-cpu-baseline --e2e-steps 0 --soak-s 0 > gpurun_out/ncu_full.log 2>&1
-python tools/ncu_summary.py gpurun_out/prof.ncu-rep > gpurun_out/ncu_full_summary.txt 2>&1
-SAFARA_LIB=$PWD/ablibs/tl.so timeout 300 python bench.py --steps 50 --warmup 5 --no-cpu-baseline --e2e-steps 0 --soak-s 0.5 > gpurun_out/tl_bench.json 2>&1
-cp gpurun_out/timeline.txt gpurun_out/timeline_full.txt
+timeout 900 python -m pytest tests -m gpu -q -x > gpurun_out/pytest_gpu.txt 2>&1
+for r in 1 2; do for v in prev cur; do echo -n "$v "; SAFARA_LIB=$PWD/ablibs/$v.so timeout 300 python bench.py --slab-sim 8 --steps 400 --warmup 10; done; done
+for p in 2 4 8; do for g in 0 20; do timeout 300 python bench.py --slab-sim $p --steps 400 --warmup 10 --graph $g; done; done
+for p in 2 4 8; do for g in 0 20; do timeout 300 python bench.py --slab-sim $p --config SP-B --steps 400 --warmup 10 --graph $g; done; done
+AB_ARGS="" bash tools/ab.sh 400 ablibs/prev.so ablibs/cur.so ablibs/prev.so ablibs/cur.so
+SAFARA_SAME_GPU=1 timeout 600 python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 --master-addr 127.0.0.1 --master-port 29533 bench.py --gpus 2 --steps 40 --warmup 3 --e2e-steps 2 --soak-s 0.2 --graph 20 > gpurun_out/dist2g.json 2>&1
