@@ -54,9 +54,12 @@ def parse():
                     help="N>1: peer = halo fused into the kernel (loads from the neighbours' "
                          "slabs over NVLink, SURVEY f2); nccl = NCCL send/recv exchange "
                          "overlapped with the interior planes (SURVEY §8(e))")
-    ap.add_argument("--graph", type=int, default=0, metavar="G",
-                    help="N=1: capture G passes into one CUDA graph and replay it K/G times "
-                         "(the per-launch gap becomes a graph-internal one)")
+    ap.add_argument("--graph", type=int, default=-1, metavar="G",
+                    help="capture G passes into one CUDA graph and replay it K/G times (the "
+                         "per-launch gap becomes a graph-internal one); default: 0 at N=1 "
+                         "(back-to-back graph replays raise the power draw and the cap takes "
+                         "it back in clock), 20 for the fused-halo multi-GPU path (per-rank "
+                         "passes of 10-20 us, where the launch gap is 10%%)")
     ap.add_argument("--slab-sim", type=int, default=0, metavar="P",
                     help="one GPU: time the middle rank's fused-halo pass of a P-way "
                          "z-split (neighbour slabs resident on the same GPU) next to the "
@@ -483,6 +486,9 @@ def run_slab_sim(args):
 
 def main():
     args = parse()
+    if args.graph < 0:
+        multi = int(os.environ.get("WORLD_SIZE", "1")) > 1 or args.gpus > 1
+        args.graph = 20 if multi and args.halo == "peer" else 0
     if args.slab_sim:
         run_slab_sim(args)
         return
