@@ -55,6 +55,8 @@ struct Tune {
     int interleave = 1;  // lockstep CTA order: 1 = tile-major across CTAs, 0 = part-major
     int face_ctas = 1;   // boundary faces on the idle SMs' extra CTAs (else by compute CTAs)
     int min_planes = MIN_PLANES_PER_CTA;  // shortest k-run a CTA is given
+    int peer_bias = 3;   // f2: planes the slab-end k-part gives up (its tail waits for a peer)
+    int split_bias = 0;  // experiments: shift the lockstep k-split points (no peer)
 } g_tune;
 
 int env_int(const char *name, int dflt) {
@@ -237,6 +239,16 @@ int launch(const double *u, const double *f, double *r, const safara_dims_t &d, 
         // same time and the second read hits L2.
         ncta = p.ncol * parts;
         p.parts = g_tune.interleave ? (int)parts : 0;
+        // f2: the k-part ending at the slab end pulls the upper peer's planes
+        // in its last two steps; give it fewer planes so it ends with the rest
+        // (measured with bench.py --slab-sim: C/8 +5.5 %, SP-B/4 +21 %, SP-B/8
+        // +7 %; applied only to short parts -- at C/4, 20 planes per part, a
+        // biased split was 27 % slower, profiles/slab_sim_r01.txt)
+        if (peer && peer->u_hi != nullptr && p.parts > 1 && p.nplanes / p.parts <= 12)
+            p.split_bias = std::min(g_tune.peer_bias, std::max(0, p.nplanes / p.parts - 2));
+        else if (p.parts > 1)
+            p.split_bias = std::max(-(int)(p.nplanes / p.parts) + 2,
+                                    std::min(g_tune.split_bias, (int)(p.nplanes / p.parts) - 2));
     } else {
         ncta = (p.units + g_tune.min_planes - 1) / g_tune.min_planes;
         ncta = std::min(ncta, max_ctas);
@@ -384,6 +396,8 @@ int safara_rhs_init(int device) {
     g_tune.interleave = env_int("SAFARA_INTERLEAVE", g_tune.interleave);
     g_tune.face_ctas = env_int("SAFARA_FACE_CTAS", g_tune.face_ctas);
     g_tune.min_planes = std::max(1, env_int("SAFARA_MIN_PLANES", g_tune.min_planes));
+    g_tune.peer_bias = std::max(0, env_int("SAFARA_PEER_BIAS", g_tune.peer_bias));
+    g_tune.split_bias = env_int("SAFARA_SPLIT_BIAS", g_tune.split_bias);
     int major = 0, minor = 0, sms = 0;
     if (cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, device) ||
         cudaDeviceGetAttribute(&minor, cudaDevAttrComputeCapabilityMinor, device) ||

@@ -1030,8 +1030,13 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensor
         // lockstep: CTA c owns column tile c % ncol, k-part c / ncol (all
         // parts of one plane band run on CTAs spread over the whole chip)
         const int c = (int)blockIdx.x, col = c % P.ncol, part = c / P.ncol;
-        ub = col * P.nplanes + (part * P.nplanes) / P.parts;
-        ue = col * P.nplanes + ((part + 1) * P.nplanes) / P.parts;
+        // split_bias: the last part is made shorter by that many planes (its
+        // final steps wait for the upper peer's planes, f2), the others share them
+        const int np = P.nplanes + P.split_bias;
+        ub = col * P.nplanes + max(0, min((part * np) / P.parts, P.nplanes));
+        ue = col * P.nplanes + (part + 1 == P.parts ? P.nplanes
+                                                     : max(0, min(((part + 1) * np) / P.parts,
+                                                                  P.nplanes)));
     } else {
         ub = split_point((int)blockIdx.x, P.units, P.ncta);
         ue = split_point((int)blockIdx.x + 1, P.units, P.ncta);

@@ -69,6 +69,7 @@ struct Params {
     int ncta;              // compute CTAs (the grid has ncta + nface_cta)
     int nface_cta;         // extra CTAs that only copy boundary faces (0: compute CTAs do it)
     int parts;             // lockstep: k-parts per column (CTA c -> tile c % ncol); 0 = ranges
+    int split_bias;        // lockstep: planes the last k-part gives to the others (f2)
     int units;             // ncol*nplanes (column-plane work items, < 2^31)
     int fk_lo, fk_hi;      // local planes whose boundary faces this launch copies
     int pos_j, pos_m, pos_k;  // tensor-map dimension holding j, m, k
