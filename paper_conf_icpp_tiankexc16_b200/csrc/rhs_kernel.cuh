@@ -58,6 +58,12 @@
 #ifndef SAFARA_PROBE
 #define SAFARA_PROBE 0  // roofline probes: 1 memory only, 2 compute only (no TMA waits/refills, no stores), 3 no rhs stores
 #endif
+#ifndef SAFARA_F_HINT
+#define SAFARA_F_HINT 0  // 1: forcing TMA loads with an L2 evict_first hint
+#endif
+#ifndef SAFARA_U_HINT
+#define SAFARA_U_HINT 0  // 1: u TMA loads with an L2 evict_last hint
+#endif
 #ifndef SAFARA_KBM_SMEM
 #define SAFARA_KBM_SMEM 1  // unchecked-march bound read from shared memory each iteration
 #endif
@@ -157,6 +163,29 @@ __device__ __forceinline__ void tma_load_4d(void *dst, const CUtensorMap *map, u
         "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(c2), "r"(c3),
         "r"(smem_u32(bar))
         : "memory");
+}
+
+// The same load with an L2 eviction-priority hint (createpolicy): forcing is
+// read exactly once, so it can leave L2 first and leave room for the u halo
+// rows that neighbouring tiles read again.
+__device__ __forceinline__ void tma_load_4d_hint(void *dst, const CUtensorMap *map, uint64_t *bar,
+                                                 int c0, int c1, int c2, int c3, uint64_t pol) {
+    asm volatile(
+        "cp.async.bulk.tensor.4d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
+        ".L2::cache_hint [%0], [%1, {%2, %3, %4, %5}], [%6], %7;" ::"r"(smem_u32(dst)),
+        "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(c2), "r"(c3),
+        "r"(smem_u32(bar)), "l"(pol)
+        : "memory");
+}
+__device__ __forceinline__ uint64_t policy_evict_first() {
+    uint64_t pol;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+    return pol;
+}
+__device__ __forceinline__ uint64_t policy_evict_last() {
+    uint64_t pol;
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
+    return pol;
 }
 
 __device__ __forceinline__ void tma_prefetch_l2_4d(const CUtensorMap *map, int c0, int c1, int c2,
@@ -605,7 +634,11 @@ __device__ __forceinline__ void issue_plane(const CUtensorMap *umap, const CUten
                     P.pos_m == 2 ? m : c2, P.pos_m == 3 ? m : c3);
     }
 #else
+#if SAFARA_U_HINT == 1
+    tma_load_4d_hint(dst, umap, &full[slot], i0 - HX, c1, c2, c3, policy_evict_last());
+#else
     tma_load_4d(dst, umap, &full[slot], i0 - HX, c1, c2, c3);
+#endif
 #endif
     if (with_f) {
         const int f1 = P.pos_j == 1 ? j0 : (P.pos_m == 1 ? 0 : kf);
@@ -616,7 +649,11 @@ __device__ __forceinline__ void issue_plane(const CUtensorMap *umap, const CUten
             tma_load_4d(dst + U_SLOT + m * FX * TY, fmap, &full[slot], i0 - 1,
                         P.pos_m == 1 ? m : f1, P.pos_m == 2 ? m : f2, P.pos_m == 3 ? m : f3);
 #else
+#if SAFARA_F_HINT == 1
+        tma_load_4d_hint(dst + U_SLOT, fmap, &full[slot], i0 - 1, f1, f2, f3, policy_evict_first());
+#else
         tma_load_4d(dst + U_SLOT, fmap, &full[slot], i0 - 1, f1, f2, f3);
+#endif
 #endif
     }
 }
