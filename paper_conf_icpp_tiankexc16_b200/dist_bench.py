@@ -55,14 +55,34 @@ def run(args):
     c = coeffs_nas(n, n, n, dt)
     comm = torch.cuda.Stream()
     compute = torch.cuda.current_stream()
-    halo = sd.PeerHalo(s) if args.halo == "peer" else None
+    def all_ok(ok: bool) -> bool:
+        """Every rank succeeded (collective agreement on a local outcome)."""
+        f = torch.tensor([0 if ok else 1], device=cdev)
+        dist.all_reduce(f, op=dist.ReduceOp.MAX)
+        return int(f.item()) == 0
+
+    halo, note = None, None
+    if args.halo == "peer":
+        # the fused halo needs CUDA IPC + peer access between the ranks' GPUs;
+        # if any rank cannot map its neighbours, every rank uses the NCCL halo
+        try:
+            halo = sd.PeerHalo(s)
+            ok = True
+        except Exception as e:  # noqa: BLE001 -- reported in the JSON line
+            ok, note = False, f"peer halo unavailable ({type(e).__name__}: {e}); NCCL halo used"
+        if not all_ok(ok):
+            if halo is not None:
+                halo.close()
+            halo = None
+            note = note or "a peer rank could not map its neighbours; NCCL halo used"
 
     use_graph = args.graph > 0 and halo is not None
+    auto_epochs = use_graph  # fixed for the run: never mix host and device epoch numbering
 
     def step(st=None):
         if halo is not None:
             # graph mode: device-counted epochs (the same struct replays)
-            sd.rhs_fused(s, halo, c, strict=args.strict, stream=st or compute, auto=use_graph)
+            sd.rhs_fused(s, halo, c, strict=args.strict, stream=st or compute, auto=auto_epochs)
         else:
             sd.rhs_sharded(s, c, comm_stream=comm, strict=args.strict)
 
@@ -74,18 +94,26 @@ def run(args):
         torch.cuda.synchronize()
         graph = torch.cuda.CUDAGraph()
         g0 = launch_count()
-        with torch.cuda.graph(graph):
-            for _ in range(args.graph):
-                step(torch.cuda.current_stream())
+        try:
+            with torch.cuda.graph(graph):
+                for _ in range(args.graph):
+                    step(torch.cuda.current_stream())
+            ok = True
+        except Exception as e:  # noqa: BLE001 -- reported in the JSON line
+            ok, note = False, f"graph capture failed ({type(e).__name__}); stream launches used"
         per_graph = launch_count() - g0
-        G = args.graph
-        args.steps = max(G, (args.steps // G) * G)
         torch.cuda.synchronize()
-        dist.barrier()
         eager_step = step
+        if all_ok(ok):
+            G = args.graph
+            args.steps = max(G, (args.steps // G) * G)
+            dist.barrier()
 
-        def step(st=None):  # noqa: F811 -- one replay = G passes
-            graph.replay()
+            def step(st=None):  # noqa: F811 -- one replay = G passes
+                graph.replay()
+        else:
+            use_graph = False
+            note = note or "graph capture failed on a peer rank; stream launches used"
 
     w0, w1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     w0.record(compute)
@@ -185,6 +213,7 @@ def run(args):
                     "note": "every rank copies its slab (u incl. ghosts, forcing) in and rhs out"},
             "gpu_launches": int(launches.item()),
             "peer_wait_timeouts": int(io[2].item()),
+            "note": note,
             "kernel": kernel_info(args.strict),
         }
         print(json.dumps(line), flush=True)
