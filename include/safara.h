@@ -164,7 +164,10 @@ int safara_rhs_slab(const double *u_slab, const double *forcing_slab,
  *                 without one.  A wait longer than ~2 s gives up and
  *                 increments flags[SAFARA_PEER_TIMEOUTS] (results are then
  *                 undefined; nothing hangs).
- * Results are bit-identical to safara_rhs_slab (same kernel body).
+ * Results: STRICT bit-identical to the oracle (as every entry point);
+ * production within the reading-c5 tolerance (the k-part split of a peer
+ * slab can differ from safara_rhs_slab's, and each unrolled step position
+ * may be FMA-contracted differently).
  * Errors: those of safara_rhs_slab, plus SAFARA_ERR_ARG (peer NULL, a
  * neighbour pointer missing / present against the grid ends, flags NULL or
  * not 8-byte aligned with epoch > 0, k0_lo / k0_hi inconsistent).          */
