@@ -55,8 +55,9 @@ struct Tune {
     int interleave = 1;  // lockstep CTA order: 1 = tile-major across CTAs, 0 = part-major
     int face_ctas = 1;   // boundary faces on the idle SMs' extra CTAs (else by compute CTAs)
     int min_planes = MIN_PLANES_PER_CTA;  // shortest k-run a CTA is given
-    int peer_bias = 3;   // f2: planes the slab-end k-part gives up (its tail waits for a peer)
+    int peer_bias = 1;   // f2: planes the slab-end k-part gives up (its tail waits for a peer)
     int split_bias = 0;  // experiments: shift the lockstep k-split points (no peer)
+    int peer_bias_maxpart = 6;  // peer_bias only for k-parts of at most this many planes
 } g_tune;
 
 int env_int(const char *name, int dflt) {
@@ -241,10 +242,11 @@ int launch(const double *u, const double *f, double *r, const safara_dims_t &d, 
         p.parts = g_tune.interleave ? (int)parts : 0;
         // f2: the k-part ending at the slab end pulls the upper peer's planes
         // in its last two steps; give it fewer planes so it ends with the rest
-        // (measured with bench.py --slab-sim: C/8 +5.5 %, SP-B/4 +21 %, SP-B/8
-        // +7 %; applied only to short parts -- at C/4, 20 planes per part, a
-        // biased split was 27 % slower, profiles/slab_sim_r01.txt)
-        if (peer && peer->u_hi != nullptr && p.parts > 1 && p.nplanes / p.parts <= 12)
+        // (bench.py --slab-sim with the single-loop march: SP-B/8 0.71 -> 0.75,
+        // SP-B/4 1.03 -> 1.05; on 10-plane parts (C/8) no bias is best,
+        // profiles/slab_sim_r01.txt)
+        if (peer && peer->u_hi != nullptr && p.parts > 1 &&
+            p.nplanes / p.parts <= g_tune.peer_bias_maxpart)
             p.split_bias = std::min(g_tune.peer_bias, std::max(0, p.nplanes / p.parts - 2));
         else if (p.parts > 1)
             p.split_bias = std::max(-(int)(p.nplanes / p.parts) + 2,
@@ -268,6 +270,34 @@ int launch(const double *u, const double *f, double *r, const safara_dims_t &d, 
                       ? (int)std::min<long long>({max_ctas - ncta, 32, (face_pts + 4095) / 4096})
                       : 0;
 
+#ifdef SAFARA_STEPLOG
+    {   // debug builds only: per-CTA step timestamps of the last launch
+        static unsigned long long *sl = nullptr;
+        static int nct2 = 0;
+        static int kaa[1024];
+        if (!sl) {
+            cudaMalloc(&sl, 1024 * 128 * sizeof(unsigned long long));
+            std::atexit([] {
+                static unsigned long long h[1024 * 128];
+                cudaDeviceSynchronize();
+                cudaMemcpy(h, sl, sizeof(h), cudaMemcpyDeviceToHost);
+                FILE *f = std::fopen("gpurun_out/steplog.txt", "w");
+                if (f) {
+                    for (int c = 0; c < nct2; ++c) {
+                        std::fprintf(f, "%d", c);
+                        for (int t = 0; t < 128; ++t) std::fprintf(f, " %llu", h[c * 128 + t]);
+                        std::fprintf(f, "\n");
+                    }
+                    std::fclose(f);
+                }
+            });
+        }
+        cudaMemsetAsync(sl, 0, 1024 * 128 * sizeof(unsigned long long), stream);
+        p.steplog = sl;
+        nct2 = p.ncta + p.nface_cta;
+        (void)kaa;
+    }
+#endif
 #ifdef SAFARA_TIMELINE
     {   // debug builds only: a static per-CTA timestamp buffer, dumped at exit
         // the last 4 launches, ring-indexed by launch number; the dump lists
@@ -398,6 +428,7 @@ int safara_rhs_init(int device) {
     g_tune.min_planes = std::max(1, env_int("SAFARA_MIN_PLANES", g_tune.min_planes));
     g_tune.peer_bias = std::max(0, env_int("SAFARA_PEER_BIAS", g_tune.peer_bias));
     g_tune.split_bias = env_int("SAFARA_SPLIT_BIAS", g_tune.split_bias);
+    g_tune.peer_bias_maxpart = env_int("SAFARA_PEER_BIAS_MAXPART", g_tune.peer_bias_maxpart);
     int major = 0, minor = 0, sms = 0;
     if (cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, device) ||
         cudaDeviceGetAttribute(&minor, cudaDevAttrComputeCapabilityMinor, device) ||

@@ -93,6 +93,7 @@ struct Params {
     unsigned long long *pflags, *pflags_lo, *pflags_hi;
     unsigned long long epoch;  // 0: none; SAFARA_PEER_EPOCH_AUTO: device counter
     unsigned long long *dbg;  // SAFARA_TIMELINE builds: per-CTA {start, end, smid}
+    unsigned long long *steplog;  // SAFARA_STEPLOG builds: per-CTA globaltimer at each step
     Coef c;
 };
 
