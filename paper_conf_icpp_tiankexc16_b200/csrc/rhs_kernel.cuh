@@ -64,12 +64,6 @@
 #ifndef SAFARA_U_HINT
 #define SAFARA_U_HINT 0  // 1: u TMA loads with an L2 evict_last hint
 #endif
-#ifndef SAFARA_ONELOOP
-// 2: slabs with an upper peer march with one checked 3-step loop (steps past
-// the end return early; no cold tail code), others with the split loops;
-// 1: always the single loop; 0: always the split loops
-#define SAFARA_ONELOOP 2
-#endif
 #ifndef SAFARA_KBM_SMEM
 #define SAFARA_KBM_SMEM 1  // unchecked-march bound read from shared memory each iteration
 #endif
@@ -801,9 +795,7 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensor
                                          const CUtensorMap *fmap, int k) {
     constexpr int Q = R % 3, Z = (R + 1) % 3, PI = (R + 2) % 3;  // planes k-1, k, k+1
     const unsigned FULL = 0xffffffffu;
-#if SAFARA_ONELOOP
-    if (PCHK && k >= g.kb) return;  // past the segment end (whole 3-step groups only)
-#endif
+    if (PCHK && k >= g.kb) return;  // single-loop march: past the segment end
 #ifdef SAFARA_STEPLOG
     if (threadIdx.x == 0 && P.steplog && k - g.ka < 126)
         P.steplog[blockIdx.x * 128 + 2 + (k - g.ka)] = global_ns();
@@ -1024,7 +1016,8 @@ __device__ __forceinline__ void rhs_step(Seg &g, const Params &P, const CUtensor
 // warp to release it).
 // UD: the host verified dX1..dX5 are equal per axis (true for NAS), so one
 // d1 coefficient per axis suffices -- fewer uniform registers to reload.
-template <bool UD, bool AUX>
+// ONE: the single-loop march (slabs with an upper peer, see below).
+template <bool UD, bool AUX, bool ONE>
 __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensorMap *fmap,
                                          const Params &P) {
 #ifdef SAFARA_TIMELINE
@@ -1217,21 +1210,18 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensor
         }
 
         int k = ka;
-#if SAFARA_ONELOOP
-        // slabs with an upper peer (f2): one warm checked 3-step body for the
-        // whole march, steps past kb return at once -- no separately compiled
-        // tail code, which runs cold (fetched from HBM: the streaming data has
-        // flushed L2) and cost C/8 slabs 2-3 us per pass
-        if (SAFARA_ONELOOP == 1 || P.u_hi != nullptr) {
+        if (ONE) {
+            // slabs with an upper peer (f2): one warm checked 3-step body for
+            // the whole march, steps past kb return at once -- no separately
+            // compiled tail code, which runs cold (fetched from HBM: the
+            // streaming data has flushed L2) and cost C/8 slabs 2-3 us a pass
 #pragma unroll 1
             for (; k < kb; k += 3) {
                 rhs_step<0, UD, AUX, true>(g, P, umap, fmap, k);
                 rhs_step<1, UD, AUX, true>(g, P, umap, fmap, k + 1);
                 rhs_step<2, UD, AUX, true>(g, P, umap, fmap, k + 2);
             }
-        }
-#endif
-#if SAFARA_ONELOOP != 1
+        } else {
         // steps whose plane k+2 is local (all of them unless the slab's upper
         // neighbour is a peer, f2) run without the peer check
 #if SAFARA_PCHK_SPLIT
@@ -1256,7 +1246,7 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensor
             rhs_step<0, UD, AUX, true>(g, P, umap, fmap, k);
             if (k + 1 < kb) rhs_step<1, UD, AUX, true>(g, P, umap, fmap, k + 1);
         }
-#endif
+        }
         g.seq0 += (uint32_t)(s_range[2] - s_range[6] + 2);  // planes ka .. kb+1
         // Segment end: every warp has consumed every plane; planes kb, kb+1
         // were never released, so clear the counters before the next segment.
