@@ -21,7 +21,10 @@
  * P2 exact-solution residual against the independently formulated
  * nasgen.exact_rhs, P3 exact-rational brute force, P4 polynomial / impulse
  * closed forms (dissipation operator = B^T B), P5 forcing affinity, P6 i<->j
- * symmetry.  The NAS constants themselves vs the NPB source: parity unpinned
+ * symmetry, P7 O(h^2) convergence to the compressible Navier-Stokes operator
+ * (tests/test_oracle_euler_pins.py: pins c1, c2, t?2 and the viscous /
+ * artificial-dissipation constant combinations).  The physical parameter
+ * values (gamma, mu, Pr, dx..dz, dssp) vs the NPB source: parity unpinned
  * (reading c2).
  */
 #ifndef NAS_ORACLE_H
