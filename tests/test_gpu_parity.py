@@ -230,3 +230,29 @@ def test_kernel_info_zero_spill():
         assert k["local_bytes"] == 0
         assert k["ctas_per_sm"] >= 1
         assert k["regs_per_thread"] <= 255
+
+
+@pytest.mark.parametrize("shape", [(49, 49, 49), (37, 45, 61)])
+def test_analytic_navier_stokes_field(shape):
+    """P7's smooth analytic gas state (O(1) gradients in every component, unlike
+    the exact-solution x noise inputs).  STRICT: bitwise.  Production: with
+    zero forcing and dt = 1 the interior is a sum of O(tx1 |U|) ~ 1e3 terms
+    cancelling to O(1), so no contraction order meets an elementwise relative
+    bound near the zeros (measured: up to 35x it); the bound there is
+    normwise per component (measured <= 7e-14).  With a NAS-scaled forcing and
+    dt (forcing = u/2, dt = 1e-3) the elementwise c5 bound holds (0.12 of it)."""
+    from test_oracle_euler_pins import conservative
+    nz, ny, nx = shape
+    z, y, x = np.meshgrid(np.linspace(0, 1, nz), np.linspace(0, 1, ny),
+                          np.linspace(0, 1, nx), indexing="ij")
+    u = conservative(x, y, z)
+    f = np.zeros_like(u)
+    o = oracle.compute_rhs(u, f, dt=1.0, threads=8)
+    assert np.array_equal(gpu_rhs(u, f, 1.0, strict=True), o)
+    g = gpu_rhs(u, f, 1.0, strict=False)
+    for m in range(5):
+        assert np.abs(g[..., m] - o[..., m]).max() <= RTOL * np.abs(o[..., m]).max()
+    f = 0.5 * u
+    o = oracle.compute_rhs(u, f, dt=1e-3, threads=8)
+    assert np.array_equal(gpu_rhs(u, f, 1e-3, strict=True), o)
+    assert_tol(gpu_rhs(u, f, 1e-3, strict=False), o)
