@@ -228,3 +228,17 @@ def test_p7_full_operator_mutants_do_not_converge(field, factor):
     e49, _ = run(49)
     ok49, _ = full_error(49)
     assert e49 > 2.0 * ok49, (field, e49, ok49)
+
+
+def test_p7_aux_are_primitive_variables_and_sound_speed():
+    """Step-0 aux on the gas state: rho_i = 1/rho, (us, vs, ws) = velocity,
+    square = rho |v|^2 / 2, qs = |v|^2 / 2, and SP's speed = sqrt(gamma p / rho),
+    the ideal-gas speed of sound (pins c1c2 = gamma (gamma - 1))."""
+    g = np.linspace(0.0, 1.0, 11)
+    z, y, x = np.meshgrid(g, g, g, indexing="ij")
+    rho, u, v, w, p = primitives(x, y, z)
+    a = oracle.compute_aux(conservative(x, y, z), naux=7)
+    q = 0.5 * (u * u + v * v + w * w)
+    for got, want in ((a[..., 0], 1.0 / rho), (a[..., 1], u), (a[..., 2], v), (a[..., 3], w),
+                      (a[..., 4], rho * q), (a[..., 5], q), (a[..., 6], np.sqrt(GAMMA * p / rho))):
+        np.testing.assert_allclose(got, want, rtol=1e-13, atol=1e-15)
