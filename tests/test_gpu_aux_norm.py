@@ -179,3 +179,27 @@ def test_sumsq_slabs_add_up():
     for k0, k1 in ((0, 7), (7, 19), (19, 29)):
         parts.append(sr.rhs_sumsq(dr[k0:k1].contiguous(), nx, nz=nz, k0=k0).cpu().numpy())
     np.testing.assert_allclose(np.sum(parts, axis=0), total, rtol=1e-13)
+
+
+@pytest.mark.parametrize("strict", [True, False])
+def test_aux_analytic_gas_state(strict):
+    """P7's analytic gas state (tests/test_oracle_euler_pins.py): the GPU aux
+    fields against the oracle (bitwise in STRICT) and SP speed against the
+    ideal-gas sound speed sqrt(gamma p / rho)."""
+    from types import SimpleNamespace
+    from test_oracle_euler_pins import GAMMA, conservative, primitives
+    nz, ny, nx = 21, 17, 45
+    z, y, x = np.meshgrid(np.linspace(0, 1, nz), np.linspace(0, 1, ny),
+                          np.linspace(0, 1, nx), indexing="ij")
+    u = conservative(x, y, z)
+    inp = SimpleNamespace(u=u, forcing=0.5 * u, dt=1e-3)
+    g_rhs, g_aux = run_aux(inp, 7, strict)
+    o_aux = oracle.compute_aux(u, naux=7, dt=inp.dt)
+    o_rhs = oracle.compute_rhs(u, inp.forcing, dt=inp.dt, threads=8)
+    if strict:
+        assert np.array_equal(g_aux, o_aux) and np.array_equal(g_rhs, o_rhs)
+    else:
+        assert_tol(g_aux, o_aux)
+        assert_tol(g_rhs, o_rhs)
+    rho, _, _, _, p = primitives(x, y, z)
+    np.testing.assert_allclose(g_aux[..., 6], np.sqrt(GAMMA * p / rho), rtol=1e-13)
