@@ -144,6 +144,40 @@ def exact_grid(nx: int, ny: int, nz: int) -> np.ndarray:
     return exact_solution(xi[None, None, :], eta[None, :, None], zeta[:, None, None])
 
 
+def nas_initialize(nx: int, ny: int, nz: int) -> np.ndarray:
+    """NPB initialize.f: the starting u of a BT/SP run, shape (nz, ny, nx, 5).
+
+    Interior: transfinite (trilinear-blended) interpolation of the six faces'
+    exact solutions, Pxi + Peta + Pzeta - Pxi*Peta - Pxi*Pzeta - Peta*Pzeta +
+    Pxi*Peta*Pzeta with Pxi = xi*E(1,eta,zeta) + (1-xi)*E(0,eta,zeta) etc.;
+    then the exact solution on the six boundary faces (input generation for
+    the f4(ii) full-step check)."""
+    dn = (1.0 / (nx - 1), 1.0 / (ny - 1), 1.0 / (nz - 1))
+    xi = (np.arange(nx, dtype=np.float64) * dn[0])[None, None, :, None]
+    eta = (np.arange(ny, dtype=np.float64) * dn[1])[None, :, None, None]
+    zeta = (np.arange(nz, dtype=np.float64) * dn[2])[:, None, None, None]
+    X, E, Z = (np.arange(nx) * dn[0])[None, None, :], (np.arange(ny) * dn[1])[None, :, None], \
+        (np.arange(nz) * dn[2])[:, None, None]
+    px0, px1 = exact_solution(0.0, E, Z), exact_solution(1.0, E, Z)
+    py0, py1 = exact_solution(X, 0.0, Z), exact_solution(X, 1.0, Z)
+    pz0, pz1 = exact_solution(X, E, 0.0), exact_solution(X, E, 1.0)
+    Pxi = xi * px1 + (1.0 - xi) * px0
+    Peta = eta * py1 + (1.0 - eta) * py0
+    Pzeta = zeta * pz1 + (1.0 - zeta) * pz0
+    u = (Pxi + Peta + Pzeta - Pxi * Peta - Pxi * Pzeta - Peta * Pzeta + Pxi * Peta * Pzeta)
+    u = np.array(np.broadcast_to(u, (nz, ny, nx, 5)), dtype=np.float64, copy=True)
+    ex = exact_grid(nx, ny, nz)
+    for sl in ((slice(None), slice(None), 0), (slice(None), slice(None), nx - 1),
+               (slice(None), 0), (slice(None), ny - 1), (0,), (nz - 1,)):
+        u[sl] = ex[sl]
+    return u
+
+
+# NPB BT verification (verify.f, class S: 12^3, dt = 0.01, 60 iterations):
+# the problem definition of the f4(ii) full-step check.
+BT_STEPS = {"S": (12, 0.010, 60)}
+
+
 def _dissipation(ue: np.ndarray, axis: int) -> np.ndarray:
     """NPB 5-case fourth-order dissipation of ``ue`` along ``axis`` (exact_rhs
     form), returned for indices 1..n-2 along that axis (others untouched = 0)."""

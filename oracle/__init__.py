@@ -24,6 +24,7 @@ import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _SRC = os.path.join(_HERE, "nas_oracle.c")
+_SRCS = [_SRC, os.path.join(_HERE, "nas_bt.c")]
 _HDR = os.path.join(_HERE, "nas_oracle.h")
 _LIB = os.path.join(_HERE, "libnas_oracle.so")
 
@@ -55,10 +56,10 @@ _lib = None
 def build(force: bool = False) -> str:
     """Compile the oracle shared library in-tree with gcc (idempotent)."""
     stale = (not os.path.exists(_LIB) or
-             os.path.getmtime(_LIB) < max(os.path.getmtime(_SRC), os.path.getmtime(_HDR)))
+             os.path.getmtime(_LIB) < max(os.path.getmtime(p) for p in _SRCS + [_HDR]))
     if force or stale:
         tmp = _LIB + f".tmp{os.getpid()}"
-        subprocess.check_call(["gcc", *CFLAGS, "-o", tmp, _SRC, "-lm"])
+        subprocess.check_call(["gcc", *CFLAGS, "-o", tmp, *_SRCS, "-lm"])
         os.replace(tmp, _LIB)
     return _LIB
 
@@ -84,6 +85,16 @@ def _load():
             lib.oracle_rhs_sumsq.restype = ctypes.c_int
             lib.oracle_seismic_dz.argtypes = [ctypes.c_int] * 3 + [dp] * 4 + [ctypes.c_double]
             lib.oracle_seismic_dz.restype = ctypes.c_int
+            cp = ctypes.POINTER(OracleConsts)
+            lib.oracle_bt_solve.argtypes = [ctypes.c_int] * 4 + [cp, dp, dp, dp]
+            lib.oracle_bt_solve.restype = ctypes.c_int
+            lib.oracle_bt_add.argtypes = [ctypes.c_int] * 3 + [dp, dp]
+            lib.oracle_bt_add.restype = ctypes.c_int
+            lib.oracle_bt_run.argtypes = [ctypes.c_int] * 3 + [cp, dp, dp, dp, dp, ctypes.c_int,
+                                                                ctypes.c_int]
+            lib.oracle_bt_run.restype = ctypes.c_int
+            lib.oracle_error_norm.argtypes = [ctypes.c_int] * 3 + [dp, dp, dp]
+            lib.oracle_error_norm.restype = ctypes.c_int
             _lib = lib
     return _lib
 
@@ -185,3 +196,71 @@ def seismic_dz(vz1: np.ndarray, vz2: np.ndarray, vz3: np.ndarray, h: float,
                                  out.ctypes.data_as(dp), float(h)) != 0:
         raise ValueError("oracle_seismic_dz: extents must be >= 2")
     return out
+
+
+# ---- the full NPB BT time step (nas_bt.c) -------------
+
+def _nas_scratch(nz: int, ny: int, nx: int, ncomp: int) -> np.ndarray:
+    return np.zeros((nz, padded(ny), padded(nx), ncomp), dtype=np.float64)
+
+
+def bt_solve(direction: int, u: np.ndarray, rhs: np.ndarray, dt: float) -> np.ndarray:
+    """NPB BT x_solve (0), y_solve (1) or z_solve (2) applied to ``rhs``
+    (logical (nz, ny, nx, 5)); the aux fields come from compute_aux(u)."""
+    nz, ny, nx, _ = u.shape
+    consts = set_constants(nx, ny, nz, dt)
+    un = to_nas(np.asarray(u, dtype=np.float64))
+    rn = to_nas(np.asarray(rhs, dtype=np.float64))
+    an = _nas_scratch(nz, ny, nx, 6)
+    dp = ctypes.POINTER(ctypes.c_double)
+    L = _load()
+    if L.oracle_compute_aux(nx, ny, nz, ctypes.byref(consts), un.ctypes.data_as(dp),
+                            an.ctypes.data_as(dp), 6) != 0:
+        raise ValueError("oracle_compute_aux failed")
+    if L.oracle_bt_solve(int(direction), nx, ny, nz, ctypes.byref(consts), un.ctypes.data_as(dp),
+                         an.ctypes.data_as(dp), rn.ctypes.data_as(dp)) != 0:
+        raise ValueError("oracle_bt_solve failed")
+    return from_nas(rn, nx, ny)
+
+
+def bt_run(u0: np.ndarray, forcing: np.ndarray, dt: float, niter: int,
+           threads: int = 1) -> tuple[np.ndarray, np.ndarray]:
+    """``niter`` NPB BT adi steps from ``u0``; returns (u, rhs of the last
+    step after the solves), logical layout."""
+    nz, ny, nx, _ = u0.shape
+    consts = set_constants(nx, ny, nz, dt)
+    un = to_nas(np.asarray(u0, dtype=np.float64))
+    fn = to_nas(np.asarray(forcing, dtype=np.float64))
+    rn = np.zeros_like(un)
+    an = _nas_scratch(nz, ny, nx, 6)
+    dp = ctypes.POINTER(ctypes.c_double)
+    if _load().oracle_bt_run(nx, ny, nz, ctypes.byref(consts), un.ctypes.data_as(dp),
+                             fn.ctypes.data_as(dp), rn.ctypes.data_as(dp), an.ctypes.data_as(dp),
+                             int(niter), int(threads)) != 0:
+        raise ValueError("oracle_bt_run failed")
+    return from_nas(un, nx, ny), from_nas(rn, nx, ny)
+
+
+def error_norm(u: np.ndarray, u_exact: np.ndarray) -> np.ndarray:
+    """NPB error_norm: per component sqrt(sum_all (u - u_exact)^2 / prod(n-2))."""
+    nz, ny, nx, _ = u.shape
+    un = to_nas(np.asarray(u, dtype=np.float64))
+    en = to_nas(np.asarray(u_exact, dtype=np.float64))
+    out = np.zeros(5, dtype=np.float64)
+    dp = ctypes.POINTER(ctypes.c_double)
+    if _load().oracle_error_norm(nx, ny, nz, un.ctypes.data_as(dp), en.ctypes.data_as(dp),
+                                 out.ctypes.data_as(dp)) != 0:
+        raise ValueError("oracle_error_norm failed")
+    return out
+
+
+def bt_verify_norms(u0: np.ndarray, forcing: np.ndarray, u_exact: np.ndarray, dt: float,
+                    niter: int, threads: int = 1) -> tuple[np.ndarray, np.ndarray]:
+    """NPB BT verify: after ``niter`` steps, xce = error_norm(u) and
+    xcr = rhs_norm(compute_rhs(u)) / dt."""
+    nz, ny, nx, _ = u0.shape
+    u, _ = bt_run(u0, forcing, dt, niter, threads)
+    xce = error_norm(u, u_exact)
+    r = compute_rhs(u, forcing, dt=dt, threads=threads)
+    xcr = np.sqrt(rhs_sumsq(r) / ((nx - 2) * (ny - 2) * (nz - 2))) / dt
+    return xce, xcr

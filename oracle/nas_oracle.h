@@ -79,4 +79,22 @@ int oracle_rhs_sumsq(int nx, int ny, int nz, const double *rhs, double *out);
 int oracle_seismic_dz(int nx, int ny, int nz, const double *vz_1, const double *vz_2,
                       const double *vz_3, double *value_dz, double h);
 
+/* ---- the rest of an NPB BT time step (nas_bt.c) ----
+ * oracle_bt_solve: x_solve (dir 0), y_solve (1) or z_solve (2) of NPB BT:
+ *   for every interior line, the 5x5 block-tridiagonal system of the
+ *   approximate factorisation, solved in place on rhs (NAS layout); aux =
+ *   oracle_compute_aux(naux = 6) of u.  Returns 0 / -1.
+ * oracle_bt_add: u += rhs at interior points (add.f).
+ * oracle_bt_run: niter NPB adi steps (compute_rhs, x/y/z_solve, add) on u in
+ *   place; rhs (5/pt) and aux (6/pt) are caller scratch in NAS layout.
+ * oracle_error_norm: NPB error_norm of u against u_exact (both NAS layout). */
+int oracle_bt_solve(int dir, int nx, int ny, int nz, const oracle_consts_t *c,
+                    const double *u, const double *aux, double *rhs);
+int oracle_bt_add(int nx, int ny, int nz, double *u, const double *rhs);
+int oracle_bt_run(int nx, int ny, int nz, const oracle_consts_t *c, double *u,
+                  const double *forcing, double *rhs, double *aux, int niter,
+                  int nthreads);
+int oracle_error_norm(int nx, int ny, int nz, const double *u, const double *u_exact,
+                      double *rms);
+
 #endif

@@ -62,6 +62,8 @@ SAFARA_PEER_ARRIVED, SAFARA_PEER_TIMEOUTS = 4, 5
 SAFARA_PEER_TIMEOUT_WORDS, SAFARA_PEER_EPOCH_WORD = 6, 7
 SAFARA_PEER_EPOCH_AUTO = 0xFFFFFFFFFFFFFFFF
 SAFARA_IPC_HANDLE_BYTES = 64
+SAFARA_UNIQUE_ID_BYTES = 128
+SAFARA_ERR_NCCL = -9
 
 _lock = threading.Lock()
 _lib = None
@@ -96,6 +98,19 @@ _SIGS = {
     "safara_rhs_sumsq": ([_dp, ctypes.POINTER(Dims), ctypes.c_int, ctypes.c_int, _dp, _dp, _dp],
                          ctypes.c_int),
     "safara_seismic_dz": ([_dp] * 4 + [ctypes.POINTER(Dims3), ctypes.c_double, _dp], ctypes.c_int),
+    "safara_rhs_rms": ([_dp, ctypes.POINTER(Dims), _dp, _dp, _dp], ctypes.c_int),
+    "safara_get_unique_id": ([ctypes.c_char_p], ctypes.c_int),
+    "safara_shard_init": ([ctypes.c_char_p, ctypes.c_int, ctypes.c_int, ctypes.c_int,
+                           ctypes.POINTER(ctypes.c_void_p)], ctypes.c_int),
+    "safara_rhs_sharded": ([_dp, _dp, _dp, _dp] + [ctypes.c_int] * 5 + [ctypes.POINTER(Coeffs), _dp],
+                           ctypes.c_int),
+    "safara_rhs_sharded_ex": ([_dp, _dp, _dp, _dp, ctypes.POINTER(Dims), ctypes.c_int, ctypes.c_int,
+                              ctypes.POINTER(Coeffs), ctypes.c_int, _dp], ctypes.c_int),
+    "safara_shard_rms": ([_dp, _dp, ctypes.POINTER(Dims), ctypes.c_int, ctypes.c_int, _dp, _dp, _dp],
+                         ctypes.c_int),
+    "safara_shard_rank": ([_dp, ctypes.POINTER(ctypes.c_int), ctypes.POINTER(ctypes.c_int)],
+                          ctypes.c_int),
+    "safara_shard_finalize": ([_dp], ctypes.c_int),
     "safara_launch_count": ([], ctypes.c_int64),
     "safara_kernel_info": ([ctypes.c_int, ctypes.POINTER(KernelInfo)], ctypes.c_int),
     "safara_strerror": ([ctypes.c_int], ctypes.c_char_p),

@@ -23,12 +23,29 @@ NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 COMMON = ARCH + ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC",
                  "-I" + INCLUDE, "-I" + CSRC]
+
+
+def _nccl_include() -> str:
+    """Directory of nccl.h for the NCCL types/prototypes of shard.cu (the
+    library itself is dlopen()ed at run time: torch's copy in a torch process)."""
+    try:
+        import nvidia.nccl as _n  # the wheel torch loads libnccl.so.2 from
+        for base in list(getattr(_n, "__path__", [])):
+            inc = os.path.join(base, "include")
+            if os.path.exists(os.path.join(inc, "nccl.h")):
+                return inc
+    except ImportError:
+        pass
+    return "/usr/include"
+
+
 UNITS = [
     ("rhs_fast.cu", ["--fmad=true", "-Xptxas", "-v"]),
     ("rhs_strict.cu", ["--fmad=false", "-Xptxas", "-v"]),
     ("norm.cu", []),
     ("seismic.cu", ["-Xptxas", "-v"]),
     ("api.cu", []),
+    ("shard.cu", ["-I" + _nccl_include()]),
 ]
 DEPS = ["rhs_kernel.cuh", "rhs_variant.inc", "safara_internal.h"]
 
@@ -60,7 +77,7 @@ def build(force: bool = False, verbose: bool = False, extra: list[str] | None = 
         ptxas_log.append(f"== {unit} {' '.join(flags)}\n{res.stdout}{res.stderr}")
         objs.append(obj)
     tmp = lib + f".tmp{os.getpid()}"
-    cmd = [NVCC, *ARCH, "-shared", "-cudart", "static", "-o", tmp, *objs]
+    cmd = [NVCC, *ARCH, "-shared", "-cudart", "static", "-o", tmp, *objs, "-ldl"]
     res = subprocess.run(cmd, capture_output=True, text=True)
     if res.returncode != 0:
         sys.stderr.write(res.stdout + res.stderr)

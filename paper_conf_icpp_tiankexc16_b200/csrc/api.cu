@@ -58,6 +58,7 @@ struct Tune {
     int peer_bias = 1;   // f2: planes the slab-end k-part gives up (its tail waits for a peer)
     int split_bias = 0;  // experiments: shift the lockstep k-split points (no peer)
     int peer_bias_maxpart = 6;  // peer_bias only for k-parts of at most this many planes
+    int peer_timeout_ms = 30000;  // f2 flag waits: give up and trap after this long
 } g_tune;
 
 int env_int(const char *name, int dflt) {
@@ -221,6 +222,7 @@ int launch(const double *u, const double *f, double *r, const safara_dims_t &d, 
         p.u_lo = peer->u_lo; p.u_hi = peer->u_hi;
         p.pflags = peer->flags; p.pflags_lo = peer->flags_lo; p.pflags_hi = peer->flags_hi;
         p.epoch = peer->epoch;
+        p.peer_timeout_ns = (unsigned long long)g_tune.peer_timeout_ms * 1000000ull;
     }
     to_coef(*coeffs, p.c);
 
@@ -371,6 +373,8 @@ int check_aux(const double *aux, long long abytes, const double *u, long long ub
 
 }  // namespace
 
+void safara::count_launches(int n) { g_launches.fetch_add(n, std::memory_order_relaxed); }
+
 extern "C" {
 
 int safara_coeffs_nas(int nx, int ny, int nz, double dt, safara_coeffs_t *out) {
@@ -429,6 +433,7 @@ int safara_rhs_init(int device) {
     g_tune.peer_bias = std::max(0, env_int("SAFARA_PEER_BIAS", g_tune.peer_bias));
     g_tune.split_bias = env_int("SAFARA_SPLIT_BIAS", g_tune.split_bias);
     g_tune.peer_bias_maxpart = env_int("SAFARA_PEER_BIAS_MAXPART", g_tune.peer_bias_maxpart);
+    g_tune.peer_timeout_ms = std::max(1, env_int("SAFARA_PEER_TIMEOUT_MS", g_tune.peer_timeout_ms));
     int major = 0, minor = 0, sms = 0;
     if (cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, device) ||
         cudaDeviceGetAttribute(&minor, cudaDevAttrComputeCapabilityMinor, device) ||
@@ -698,8 +703,9 @@ int safara_rhs_host(const double *u_host, const double *forcing_host, double *rh
 
 int safara_norm_work_doubles(void) { return 5 * norm_grid(); }
 
-int safara_rhs_sumsq(const double *rhs, const safara_dims_t *dims, int k0, int nzl, double *work,
-                     double *out, void *stream) {
+// Shared by safara_rhs_sumsq / safara_rhs_rms: npts > 0 finishes rhs_norm.
+static int sumsq_launch(const double *rhs, const safara_dims_t *dims, int k0, int nzl,
+                        double *work, double *out, void *stream, double npts) {
     int dev;
     int rc = current_device(&dev);
     if (rc) return rc;
@@ -717,10 +723,22 @@ int safara_rhs_sumsq(const double *rhs, const safara_dims_t *dims, int k0, int n
     const int lo = std::max(k0, 1), hi = std::min(k0 + nzl, dims->nz - 1);
     const int nk = std::max(0, hi - lo);
     cudaError_t e = launch_sumsq(rhs, dims->nx, dims->ny, dims->sy, dims->sm, dims->sk, lo - k0,
-                                 nk, work, out, (cudaStream_t)stream);
+                                 nk, work, out, (cudaStream_t)stream, npts);
     if (e != cudaSuccess) return SAFARA_ERR_CUDA;
     g_launches.fetch_add(2, std::memory_order_relaxed);
     return SAFARA_OK;
+}
+
+int safara_rhs_sumsq(const double *rhs, const safara_dims_t *dims, int k0, int nzl, double *work,
+                     double *out, void *stream) {
+    return sumsq_launch(rhs, dims, k0, nzl, work, out, stream, 0.0);
+}
+
+int safara_rhs_rms(const double *rhs, const safara_dims_t *dims, double *work, double *rms,
+                   void *stream) {
+    if (!dims) return SAFARA_ERR_ARG;
+    const double npts = (double)(dims->nx - 2) * (double)(dims->ny - 2) * (double)(dims->nz - 2);
+    return sumsq_launch(rhs, dims, 0, dims->nz, work, rms, stream, npts);
 }
 
 int safara_seismic_dz(const double *vz1, const double *vz2, const double *vz3, double *value_dz,
@@ -783,6 +801,7 @@ const char *safara_strerror(int code) {
         case SAFARA_ERR_NOT_INIT: return "safara_rhs_init was not called for the current device";
         case SAFARA_ERR_CUDA: return "CUDA runtime or driver error";
         case SAFARA_ERR_NO_DEVICE: return "no sm_100 device at this index";
+        case SAFARA_ERR_NCCL: return "NCCL error (library not loadable, communicator or P2P failure)";
         default: return "unknown error code";
     }
 }

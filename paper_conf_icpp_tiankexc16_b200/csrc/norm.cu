@@ -1,8 +1,9 @@
 // norm.cu -- SURVEY §8(f) f1: the NAS rhs_norm numerator, Σ rhs(m,i,j,k)^2
 // over the interior points (1 <= i <= nx-2, 1 <= j <= ny-2, 1 <= k <= nz-2)
 // of a field in the shared `dim` layout, per component m.  NPB error.f
-// rhs_norm then takes sqrt(sum / ((nx-2)(ny-2)(nz-2))) -- done by the caller
-// after summing the slabs (an all-reduce across ranks for z-slabs).
+// rhs_norm then takes sqrt(sum / ((nx-2)(ny-2)(nz-2))): fused into the final
+// pass for a full grid (safara_rhs_rms), or a separate 1-thread-per-component
+// kernel after the cross-slab NCCL all-reduce (safara_shard_rms).
 //
 // HBM-bound streaming reduction: each warp owns whole (m, k, j) rows, lanes
 // stride i (coalesced 256 B per load), fp64 accumulation.  Deterministic: a
@@ -54,14 +55,23 @@ sumsq_partial(const double *__restrict__ rhs, int nx, int ny, int sy, int sm, in
     }
 }
 
-// one block: warp m sums component m's G partials in a fixed order
-__global__ void sumsq_final(const double *__restrict__ work, int G, double *__restrict__ out) {
+// one block: warp m sums component m's G partials in a fixed order; with
+// npts > 0 it also finishes NPB rhs_norm: out[m] = sqrt(sum / npts)
+__global__ void sumsq_final(const double *__restrict__ work, int G, double *__restrict__ out,
+                            double npts) {
     const int m = threadIdx.x / 32, lane = threadIdx.x % 32;
     if (m >= 5) return;
     double t = 0.0;
     for (int b = lane; b < G; b += 32) t += work[m * G + b];
     t = warp_sum(t);
-    if (lane == 0) out[m] = t;
+    if (lane == 0) out[m] = npts > 0.0 ? sqrt(t / npts) : t;
+}
+
+// NPB error.f rhs_norm's last step on summed numerators (after the
+// cross-slab all-reduce): v[m] = sqrt(v[m] / npts)
+__global__ void rms_finish(double *__restrict__ v, double npts) {
+    const int m = threadIdx.x;
+    if (m < 5) v[m] = sqrt(v[m] / npts);
 }
 
 }  // namespace
@@ -69,12 +79,17 @@ __global__ void sumsq_final(const double *__restrict__ work, int G, double *__re
 int norm_grid() { return 148 * 4; }
 
 cudaError_t launch_sumsq(const double *rhs, int nx, int ny, int sy, int sm, int sk, int kl0, int nk,
-                         double *work, double *out, cudaStream_t s) {
+                         double *work, double *out, cudaStream_t s, double npts) {
     const int G = norm_grid();
     sumsq_partial<<<dim3(G, 5), NORM_THREADS, 0, s>>>(rhs, nx, ny, sy, sm, sk, kl0, nk, work);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return e;
-    sumsq_final<<<1, 5 * 32, 0, s>>>(work, G, out);
+    sumsq_final<<<1, 5 * 32, 0, s>>>(work, G, out, npts);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_rms_finish(double *v, double npts, cudaStream_t s) {
+    rms_finish<<<1, 32, 0, s>>>(v, npts);
     return cudaGetLastError();
 }
 

@@ -247,8 +247,12 @@ __device__ __forceinline__ void peer_epoch_init(const Params &P) {
                       : P.epoch;
 }
 
-// Acquire flag word `word` of this rank >= epoch (bounded wait: after ~2 s
-// count a timeout and go on, so a broken peer can never hang the GPU).
+// Acquire flag word `word` of this rank >= epoch.  Bounded wait: after
+// P.peer_timeout_ns (SAFARA_PEER_TIMEOUT_MS, default 30 s) the wait is
+// recorded in the flag words and the kernel TRAPS -- the caller's next
+// synchronisation fails (cudaErrorLaunchFailure) instead of returning an rhs
+// computed from a neighbour's stale planes, and a broken peer never hangs the
+// GPU.
 __device__ __forceinline__ void peer_wait(const Params &P, int word) {
     const unsigned long long e = peer_epoch();
     const unsigned long long *f = P.pflags + word;
@@ -256,10 +260,11 @@ __device__ __forceinline__ void peer_wait(const Params &P, int word) {
     const unsigned long long t0 = global_ns();
     while (ld_acquire_sys(f) < e) {
         __nanosleep(200);
-        if (global_ns() - t0 > 2000000000ull) {
+        if (global_ns() - t0 > P.peer_timeout_ns) {
             atomicAdd(P.pflags + SAFARA_PEER_TIMEOUTS, 1ull);
             atomicOr(P.pflags + SAFARA_PEER_TIMEOUT_WORDS, 1ull << word);  // which wait
-            return;
+            __threadfence_system();
+            __trap();
         }
     }
 }
@@ -1031,6 +1036,9 @@ __device__ __forceinline__ void rhs_body(const CUtensorMap *umap, const CUtensor
     // idle) only copy the boundary faces.
     grid_dep_launch();
     if (P.epoch) {
+        // after the previous grid (PDL): its writes to u are complete before
+        // READY is published, and its epoch advance is visible
+        grid_dep_wait();
         peer_epoch_init(P);
         __syncthreads();
         peer_publish(P);

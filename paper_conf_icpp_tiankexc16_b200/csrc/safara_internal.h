@@ -92,6 +92,7 @@ struct Params {
     // (SAFARA_PEER_* indices), pflags_lo / pflags_hi = the neighbours'.
     unsigned long long *pflags, *pflags_lo, *pflags_hi;
     unsigned long long epoch;  // 0: none; SAFARA_PEER_EPOCH_AUTO: device counter
+    unsigned long long peer_timeout_ns;  // bounded flag waits, then __trap()
     unsigned long long *dbg;  // SAFARA_TIMELINE builds: per-CTA {start, end, smid}
     unsigned long long *steplog;  // SAFARA_STEPLOG builds: per-CTA globaltimer at each step
     Coef c;
@@ -106,8 +107,13 @@ cudaError_t launch_rhs_strict(const CUtensorMap &umap, const CUtensorMap &fmap, 
                               bool uniform_d, cudaStream_t s);
 // norm.cu: per-component sums of squares over interior points (f1)
 int norm_grid();
+// npts > 0: finish NPB rhs_norm in the same launch, out[m] = sqrt(sum/npts)
 cudaError_t launch_sumsq(const double *rhs, int nx, int ny, int sy, int sm, int sk, int kl0, int nk,
-                         double *work, double *out, cudaStream_t s);
+                         double *work, double *out, cudaStream_t s, double npts = 0.0);
+// v[m] = sqrt(v[m] / npts), m < 5 (rhs_norm after a cross-slab all-reduce)
+cudaError_t launch_rms_finish(double *v, double npts, cudaStream_t s);
+// api.cu: the launch counter behind safara_launch_count
+void count_launches(int n);
 
 // seismic.cu: PAPER.md Fig. 8 dz loop (f4)
 cudaError_t launch_seismic_dz(const double *vz1, const double *vz2, const double *vz3, double *out,

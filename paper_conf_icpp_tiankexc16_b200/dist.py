@@ -7,10 +7,13 @@ plane k0+t, planes 0-1 / nzl+2..nzl+3 are ghosts filled by the halo exchange
 and rhs slabs are rank-local (nzl planes).  The only communication on the path
 is this point-to-point exchange; there is no collective.
 
-The exchange uses torch.distributed P2P (NCCL over NVLink on GPUs, gloo on CPU
-for tests).  `rhs_sharded` overlaps it with the ghost-independent planes:
-PART_INTERIOR runs on the compute stream while the exchange is in flight,
-PART_EDGE after the exchange completes.
+The exchange is library code (include/safara.h safara_rhs_sharded): the
+library owns an NCCL communicator (`NcclShard`: torch supplies only the process
+group that broadcasts the NCCL unique id) and, per pass, runs the grouped
+ncclSend/ncclRecv on its comm stream while PART_INTERIOR runs on the caller's
+stream, joins, then runs PART_EDGE.  `halo_ops` / `halo_exchange` are the same
+exchange pattern written with torch.distributed P2P; they exist for the CPU
+(gloo) tests of the partition / neighbour logic.
 
 SURVEY §8(f) f2, `rhs_fused`: no exchange at all.  The only values a slab
 needs from a neighbour are the own (i, j) columns of the two planes beyond its
@@ -27,8 +30,7 @@ from dataclasses import dataclass
 import torch
 import torch.distributed as dist
 
-from ._abi import (SAFARA_PART_EDGE, SAFARA_PART_INTERIOR, SAFARA_PEER_EPOCH_AUTO,
-                   SAFARA_PEER_WORDS, Peer)
+from ._abi import SAFARA_PEER_EPOCH_AUTO, SAFARA_PEER_WORDS, Peer
 
 GHOST = 2
 
@@ -99,23 +101,51 @@ def halo_exchange(s: Slab, group=None) -> list:
     return dist.batch_isend_irecv(ops) if ops else []
 
 
-def rhs_sharded(s: Slab, coeffs, comm_stream: torch.cuda.Stream | None = None,
-                strict: bool = False, group=None) -> torch.Tensor:
-    """One distributed pass: exchange overlapped with the interior planes."""
-    from .rhs import rhs_slab
-    compute = torch.cuda.current_stream()
-    comm = comm_stream or torch.cuda.Stream()
-    comm.wait_stream(compute)  # u is ready
-    with torch.cuda.stream(comm):
-        works = halo_exchange(s, group)
-    rhs_slab(s.u, s.forcing, s.rhs, s.nx, s.nz, s.k0, coeffs, part=SAFARA_PART_INTERIOR,
-             strict=strict, stream=compute)
-    for w in works:
-        w.wait()                # compute stream waits for the ghosts
-    compute.wait_stream(comm)
-    rhs_slab(s.u, s.forcing, s.rhs, s.nx, s.nz, s.k0, coeffs, part=SAFARA_PART_EDGE,
-             strict=strict, stream=compute)
-    return s.rhs
+def broadcast_unique_id(rank: int, group=None, src: int = 0) -> bytes:
+    """Rank ``src`` draws a fresh NCCL unique id through the library
+    (safara_get_unique_id); every rank gets the same bytes through the torch
+    process group (any backend: gloo on CPU, NCCL on GPUs)."""
+    from .rhs import get_unique_id
+    obj = [get_unique_id() if rank == src else None]
+    dist.broadcast_object_list(obj, src=src, group=group)
+    return obj[0]
+
+
+class NcclShard:
+    """This rank's library-owned NCCL communicator (safara_shard_init).
+
+    torch.distributed is used once, to broadcast the unique id; every pass
+    then runs through the C ABI (safara_rhs_sharded / safara_shard_rms)."""
+
+    def __init__(self, rank: int, world: int, device: int, group=None):
+        from .rhs import init, shard_init
+        init(device)
+        uid = broadcast_unique_id(rank, group)
+        self.rank, self.world, self.device = rank, world, device
+        self.handle = shard_init(uid, rank, world, device)
+
+    def rhs(self, s: Slab, coeffs, strict: bool = False, stream=None) -> torch.Tensor:
+        from .rhs import rhs_sharded as _rhs_sharded
+        return _rhs_sharded(self.handle, s.u, s.forcing, s.rhs, s.nx, s.nz, s.k0, coeffs,
+                            strict=strict, stream=stream)
+
+    def rms(self, s: Slab, stream=None) -> torch.Tensor:
+        from .rhs import shard_rms
+        return shard_rms(self.handle, s.rhs, s.nx, s.nz, s.k0, stream=stream)
+
+    def close(self):
+        if self.handle:
+            from .rhs import shard_finalize
+            shard_finalize(self.handle)
+            self.handle = 0
+
+
+def rhs_sharded(s: Slab, coeffs, shard: NcclShard, strict: bool = False,
+                stream=None) -> torch.Tensor:
+    """One distributed pass through the library (safara_rhs_sharded): NCCL
+    halo exchange on the shard's comm stream overlapped with the interior
+    planes, then the edge planes."""
+    return shard.rhs(s, coeffs, strict=strict, stream=stream)
 
 
 # ---- SURVEY §8(f) f2: the halo fused into the pass --------------------------
@@ -155,6 +185,23 @@ def new_flags(device) -> torch.Tensor:
     return torch.zeros(SAFARA_PEER_WORDS, dtype=torch.int64, device=device)
 
 
+class PeerHaloUnavailable(RuntimeError):
+    """The fused peer halo cannot map a neighbour's slab (e.g. expandable
+    segments): use the library's NCCL path (NcclShard / rhs_sharded)."""
+
+
+def ipc_unavailable_reason() -> str:
+    """Why cudaIpcGetMemHandle may refuse torch's allocations."""
+    import os
+    conf = os.environ.get("PYTORCH_CUDA_ALLOC_CONF", "") + os.environ.get(
+        "PYTORCH_ALLOC_CONF", "")
+    if "expandable_segments:True" in conf.replace(" ", ""):
+        return ("PYTORCH_CUDA_ALLOC_CONF has expandable_segments:True: the caching allocator "
+                "maps VMM segments, which CUDA IPC cannot export; unset it or use the NCCL halo")
+    return ("the tensor is not in an IPC-exportable cudaMalloc allocation (VMM / expandable "
+            "segment or a foreign allocator); use the NCCL halo")
+
+
 class PeerHalo:
     """Peer mapping of the neighbours' u slabs and flag words (one per rank).
 
@@ -164,14 +211,23 @@ class PeerHalo:
     (epoch + 1; ``sync=False`` -> epoch 0, inputs static)."""
 
     def __init__(self, s: Slab, group=None):
+        from ._abi import SafaraError
         from .rhs import ipc_get, ipc_open
         self.slab = s
         self.flags = new_flags(s.u.device)
         self.nb = neighbours(s.nz, s.world, s.rank)
-        mine = (ipc_get(s.u), ipc_get(self.flags))
+        self._opened = []
+        # Every rank reports success or its reason, so a rank that cannot
+        # export never leaves the others blocked in the gather: all raise.
+        try:
+            mine = (ipc_get(s.u), ipc_get(self.flags))
+        except SafaraError as e:
+            mine = f"rank {s.rank}: {e} -- {ipc_unavailable_reason()}"
         allx = [None] * s.world
         dist.all_gather_object(allx, mine, group=group)
-        self._opened = []
+        bad = [x for x in allx if isinstance(x, str)]
+        if bad:
+            raise PeerHaloUnavailable("; ".join(bad))
 
         def open_(r):
             (hu, ou), (hf, of) = allx[r]

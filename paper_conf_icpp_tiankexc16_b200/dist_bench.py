@@ -2,8 +2,9 @@
 split into z-slabs, one compute_rhs pass per step.  --halo peer (default):
 the halo is fused into the kernel (safara_rhs_peer: one
 launch per rank per pass, neighbours' planes loaded over NVLink, epoch flags);
---halo nccl: NCCL send/recv exchange overlapped with the interior planes
-(SURVEY §8(e)).
+--halo nccl: the library's NCCL send/recv exchange overlapped with the
+interior planes (safara_rhs_sharded on a library-owned communicator, SURVEY
+§8(b)/(e)).
 
 Timing: barrier + synchronize on both sides of the K timed steps, CUDA events
 on each rank's compute stream, MAX over ranks (all_reduce).  value = all grid
@@ -53,7 +54,6 @@ def run(args):
     ug, fg = pack(inp.u, device="cpu"), pack(inp.forcing, device="cpu")
     s = sd.make_slab(ug, fg, n, rank, world, device=f"cuda:{local}")
     c = coeffs_nas(n, n, n, dt)
-    comm = torch.cuda.Stream()
     compute = torch.cuda.current_stream()
     def all_ok(ok: bool) -> bool:
         """Every rank succeeded (collective agreement on a local outcome)."""
@@ -76,6 +76,11 @@ def run(args):
             halo = None
             note = note or "a peer rank could not map its neighbours; NCCL halo used"
 
+    shard = None
+    if halo is None:
+        # the library owns the communicator; torch only broadcasts its id
+        shard = sd.NcclShard(rank, world, local)
+
     use_graph = args.graph > 0 and halo is not None
     auto_epochs = use_graph  # fixed for the run: never mix host and device epoch numbering
 
@@ -84,7 +89,7 @@ def run(args):
             # graph mode: device-counted epochs (the same struct replays)
             sd.rhs_fused(s, halo, c, strict=args.strict, stream=st or compute, auto=auto_epochs)
         else:
-            sd.rhs_sharded(s, c, comm_stream=comm, strict=args.strict)
+            sd.rhs_sharded(s, c, shard, strict=args.strict, stream=st or compute)
 
     if use_graph:
         # G passes per CUDA graph (one launch gap per G passes); every rank
@@ -183,6 +188,9 @@ def run(args):
         torch.cuda.synchronize()
         dist.barrier()          # nobody unmaps a slab a neighbour may still read
         halo.close()
+    if shard is not None:
+        torch.cuda.synchronize()
+        shard.close()
 
     if rank == 0:
         peak, peak_kind = measured_peaks()
@@ -198,7 +206,8 @@ def run(args):
                                        "peer loads, epoch flags)" + (
                                            f", CUDA graph of {args.graph} passes" if use_graph
                                            else "") if halo is not None else
-                                       f"z-slab x{world}, 2-plane NCCL send/recv halo"),
+                                       f"z-slab x{world}, 2-plane NCCL send/recv halo "
+                                       "(library-owned communicator)"),
                        "variant": "strict" if args.strict else "production",
                        "l2": "per-rank slabs; inputs > L2 at C/1-2, no flush"},
             "hbm_gbs": achieved,

@@ -14,7 +14,8 @@ import numpy as np
 import torch
 
 from ._abi import (SAFARA_AUX_BT, SAFARA_AUX_SP, SAFARA_FLAG_STRICT, SAFARA_IPC_HANDLE_BYTES,
-                   SAFARA_PART_ALL, Coeffs, Dims, Dims3, KernelInfo, Peer, check, lib)
+                   SAFARA_PART_ALL, SAFARA_UNIQUE_ID_BYTES, Coeffs, Dims, Dims3, KernelInfo, Peer,
+                   check, lib)
 
 _initialised: set[int] = set()
 
@@ -85,17 +86,59 @@ def _check_field(t: torch.Tensor, name: str):
         raise ValueError(f"{name} must be a contiguous float64 CUDA tensor")
 
 
+def _check_shape(t: torch.Tensor, shape: tuple, name: str):
+    """The C side sizes its TMA maps and stores from the descriptor alone, so
+    every tensor must really hold the planes the descriptor implies."""
+    if tuple(t.shape) != tuple(shape):
+        raise ValueError(f"{name} has shape {tuple(t.shape)}, expected {tuple(shape)}")
+
+
+def _max_offset(d: Dims, nplanes: int, ncomp: int = 5) -> int:
+    return (d.nx - 1) + d.sy * (d.ny - 1) + d.sm * (ncomp - 1) + d.sk * (nplanes - 1)
+
+
+def _check_numel(t: torch.Tensor, d: Dims, nplanes: int, name: str):
+    need = _max_offset(d, nplanes) + 1
+    if t.numel() < need:
+        raise ValueError(f"{name} holds {t.numel()} doubles, the descriptor reaches {need}")
+
+
+def _canonical_fields(nx: int, fields, nplanes_u: int | None = None):
+    """Check canonical (nplanes, 5, ny, pitch(nx)) tensors: fields[0] is u
+    (nplanes_u planes if given, else the same as the others)."""
+    ref = fields[1][0]
+    nzl, five, ny, sy = ref.shape if ref.dim() == 4 else (None, None, None, None)
+    if ref.dim() != 4 or five != 5 or sy != pitch(nx):
+        raise ValueError(f"{fields[1][1]} must be canonical (nplanes, 5, ny, {pitch(nx)}), "
+                         f"got {tuple(ref.shape)}")
+    for i, (t, n) in enumerate(fields):
+        want = (nplanes_u if (i == 0 and nplanes_u is not None) else nzl, 5, ny, sy)
+        _check_shape(t, want, n)
+    return nzl, ny
+
+
 def rhs(u: torch.Tensor, forcing: torch.Tensor, out: torch.Tensor, nx: int, coeffs: Coeffs,
         strict: bool = False, stream=None, dims: Dims | None = None) -> torch.Tensor:
     """One compute_rhs pass: ``out <- F(u, forcing)`` on the GPU (async).
 
     Tensors are canonical ``(nz, 5, ny, sy)`` unless ``dims`` describes
-    another stride order (then they are flat buffers of that layout)."""
+    another stride order (then they are flat buffers of that layout).
+    Canonical + production calls ``safara_rhs`` itself; STRICT or an explicit
+    descriptor goes through ``safara_rhs_ex``."""
     for t, n in ((u, "u"), (forcing, "forcing"), (out, "out")):
         _check_field(t, n)
     if dims is None:
-        nz, _, ny, _ = u.shape
+        nz, ny = _canonical_fields(nx, ((u, "u"), (forcing, "forcing"), (out, "out")))
+        if not strict:
+            # the north_star entry point itself: canonical layout, production
+            check(lib().safara_rhs(u.data_ptr(), forcing.data_ptr(), out.data_ptr(), int(nx),
+                                   int(ny), int(nz), ctypes.byref(coeffs), _stream_ptr(stream)),
+                  "safara_rhs")
+            return out
         dims = canonical_dims(nx, ny, nz)
+    else:
+        for t, n in ((u, "u"), (forcing, "forcing"), (out, "out")):
+            _check_numel(t, dims, dims.nz, n)
     flags = SAFARA_FLAG_STRICT if strict else 0
     check(lib().safara_rhs_ex(u.data_ptr(), forcing.data_ptr(), out.data_ptr(),
                               ctypes.byref(dims), ctypes.byref(coeffs), flags,
@@ -110,7 +153,9 @@ def rhs_slab(u_slab: torch.Tensor, forcing_slab: torch.Tensor, out_slab: torch.T
     out have nzl planes; this slab owns global planes [k0, k0+nzl)."""
     for t, n in ((u_slab, "u_slab"), (forcing_slab, "forcing_slab"), (out_slab, "out_slab")):
         _check_field(t, n)
-    nzl, _, ny, _ = forcing_slab.shape
+    nzl = forcing_slab.shape[0]
+    _, ny = _canonical_fields(nx, ((u_slab, "u_slab"), (forcing_slab, "forcing_slab"),
+                                   (out_slab, "out_slab")), nplanes_u=nzl + 4)
     dims = canonical_dims(nx, ny, nz)
     flags = SAFARA_FLAG_STRICT if strict else 0
     check(lib().safara_rhs_slab(u_slab.data_ptr(), forcing_slab.data_ptr(), out_slab.data_ptr(),
@@ -127,7 +172,9 @@ def rhs_peer(u_slab: torch.Tensor, forcing_slab: torch.Tensor, out_slab: torch.T
     exchange.  Slab tensors as in :func:`rhs_slab` (ghost planes unused)."""
     for t, n in ((u_slab, "u_slab"), (forcing_slab, "forcing_slab"), (out_slab, "out_slab")):
         _check_field(t, n)
-    nzl, _, ny, _ = forcing_slab.shape
+    nzl = forcing_slab.shape[0]
+    _, ny = _canonical_fields(nx, ((u_slab, "u_slab"), (forcing_slab, "forcing_slab"),
+                                   (out_slab, "out_slab")), nplanes_u=nzl + 4)
     dims = canonical_dims(nx, ny, nz)
     flags = SAFARA_FLAG_STRICT if strict else 0
     check(lib().safara_rhs_peer(u_slab.data_ptr(), forcing_slab.data_ptr(), out_slab.data_ptr(),
@@ -135,6 +182,76 @@ def rhs_peer(u_slab: torch.Tensor, forcing_slab: torch.Tensor, out_slab: torch.T
                                 ctypes.byref(coeffs), flags, _stream_ptr(stream)),
           "safara_rhs_peer")
     return out_slab
+
+
+# ---- the sharded pass, library-owned NCCL communicator ----
+
+def get_unique_id() -> bytes:
+    """safara_get_unique_id: SAFARA_UNIQUE_ID_BYTES opaque bytes (rank 0)."""
+    b = ctypes.create_string_buffer(SAFARA_UNIQUE_ID_BYTES)
+    check(lib().safara_get_unique_id(b), "safara_get_unique_id")
+    return b.raw
+
+
+def shard_init(uid: bytes, rank: int, nranks: int, device: int) -> int:
+    """safara_shard_init; returns the opaque shard handle (an address)."""
+    if len(uid) != SAFARA_UNIQUE_ID_BYTES:
+        raise ValueError(f"unique id must be {SAFARA_UNIQUE_ID_BYTES} bytes")
+    h = ctypes.c_void_p()
+    check(lib().safara_shard_init(uid, int(rank), int(nranks), int(device), ctypes.byref(h)),
+          "safara_shard_init")
+    return int(h.value)
+
+
+def shard_finalize(handle: int) -> None:
+    check(lib().safara_shard_finalize(handle), "safara_shard_finalize")
+
+
+def shard_rank(handle: int) -> tuple[int, int]:
+    r, n = ctypes.c_int(), ctypes.c_int()
+    check(lib().safara_shard_rank(handle, ctypes.byref(r), ctypes.byref(n)), "safara_shard_rank")
+    return r.value, n.value
+
+
+def rhs_sharded(handle: int, u_slab: torch.Tensor, forcing_slab: torch.Tensor,
+                out_slab: torch.Tensor, nx: int, nz: int, k0: int, coeffs: Coeffs,
+                strict: bool = False, stream=None) -> torch.Tensor:
+    """safara_rhs_sharded(_ex): NCCL halo exchange into u_slab's ghost planes
+    overlapped with the interior planes, then the edge planes (async)."""
+    for t, n in ((u_slab, "u_slab"), (forcing_slab, "forcing_slab"), (out_slab, "out_slab")):
+        _check_field(t, n)
+    nzl = forcing_slab.shape[0]
+    _, ny = _canonical_fields(nx, ((u_slab, "u_slab"), (forcing_slab, "forcing_slab"),
+                                   (out_slab, "out_slab")), nplanes_u=nzl + 4)
+    L = lib()
+    if strict:
+        dims = canonical_dims(nx, ny, nz)
+        rc = L.safara_rhs_sharded_ex(handle, u_slab.data_ptr(), forcing_slab.data_ptr(),
+                                     out_slab.data_ptr(), ctypes.byref(dims), int(k0), int(nzl),
+                                     ctypes.byref(coeffs), SAFARA_FLAG_STRICT, _stream_ptr(stream))
+        check(rc, "safara_rhs_sharded_ex")
+    else:
+        rc = L.safara_rhs_sharded(handle, u_slab.data_ptr(), forcing_slab.data_ptr(),
+                                  out_slab.data_ptr(), int(nx), int(ny), int(nz), int(k0),
+                                  int(nzl), ctypes.byref(coeffs), _stream_ptr(stream))
+        check(rc, "safara_rhs_sharded")
+    return out_slab
+
+
+def shard_rms(handle: int, r_slab: torch.Tensor, nx: int, nz: int, k0: int, stream=None,
+              out: torch.Tensor | None = None) -> torch.Tensor:
+    """safara_shard_rms: NPB rhs_norm over every rank's slab (NCCL all-reduce
+    of the per-slab sums, finished on the device); 5 device doubles (async)."""
+    _check_field(r_slab, "rhs_slab")
+    nzl, ny = _canonical_fields(nx, ((r_slab, "rhs_slab"), (r_slab, "rhs_slab")))
+    dims = canonical_dims(nx, ny, nz)
+    work = _work_for(r_slab, stream)
+    if out is None:
+        out = torch.empty(5, dtype=torch.float64, device=r_slab.device)
+    check(lib().safara_shard_rms(handle, r_slab.data_ptr(), ctypes.byref(dims), int(k0), int(nzl),
+                                 work.data_ptr(), out.data_ptr(), _stream_ptr(stream)),
+          "safara_shard_rms")
+    return out
 
 
 def ipc_get(t: torch.Tensor) -> tuple[bytes, int]:
@@ -160,7 +277,10 @@ def rhs_host(u_host: torch.Tensor, f_host: torch.Tensor, r_host: torch.Tensor,
              u_dev: torch.Tensor, f_dev: torch.Tensor, r_dev: torch.Tensor, nx: int,
              coeffs: Coeffs, strict: bool = False, nchunks: int = 8, stream=None):
     """End-to-end pass on host (pinned) canonical tensors through device buffers."""
-    nz, _, ny, _ = u_host.shape
+    nz, ny = _canonical_fields(nx, ((u_host, "u_host"), (f_host, "f_host"), (r_host, "r_host")))
+    for t, n in ((u_dev, "u_dev"), (f_dev, "f_dev"), (r_dev, "r_dev")):
+        _check_field(t, n)
+        _check_shape(t, tuple(u_host.shape), n)
     flags = SAFARA_FLAG_STRICT if strict else 0
     check(lib().safara_rhs_host(u_host.data_ptr(), f_host.data_ptr(), r_host.data_ptr(),
                                 u_dev.data_ptr(), f_dev.data_ptr(), r_dev.data_ptr(),
@@ -204,8 +324,14 @@ def rhs_aux(u: torch.Tensor, forcing: torch.Tensor, out: torch.Tensor, aux: torc
     for t, n in ((u, "u"), (forcing, "forcing"), (out, "out"), (aux, "aux")):
         _check_field(t, n)
     if dims is None:
-        nz, _, ny, _ = u.shape
+        nz, ny = _canonical_fields(nx, ((u, "u"), (forcing, "forcing"), (out, "out")))
         dims = canonical_dims(nx, ny, nz)
+        if aux.dim() != 4 or aux.shape[1] not in (SAFARA_AUX_BT, SAFARA_AUX_SP):
+            raise ValueError(f"aux must be (nz, 6|7, ny, sy), got {tuple(aux.shape)}")
+        _check_shape(aux, (nz, aux.shape[1], ny, pitch(nx)), "aux")
+    else:
+        for t, n in ((u, "u"), (forcing, "forcing"), (out, "out")):
+            _check_numel(t, dims, dims.nz, n)
     naux = int(aux.shape[1]) if aux.dim() == 4 else SAFARA_AUX_BT
     flags = SAFARA_FLAG_STRICT if strict else 0
     check(lib().safara_rhs_aux(u.data_ptr(), forcing.data_ptr(), out.data_ptr(), aux.data_ptr(),
@@ -220,7 +346,12 @@ def rhs_slab_aux(u_slab, forcing_slab, out_slab, aux_slab, nx: int, nz: int, k0:
     for t, n in ((u_slab, "u_slab"), (forcing_slab, "forcing_slab"), (out_slab, "out_slab"),
                  (aux_slab, "aux_slab")):
         _check_field(t, n)
-    nzl, _, ny, _ = forcing_slab.shape
+    nzl = forcing_slab.shape[0]
+    _, ny = _canonical_fields(nx, ((u_slab, "u_slab"), (forcing_slab, "forcing_slab"),
+                                   (out_slab, "out_slab")), nplanes_u=nzl + 4)
+    if aux_slab.dim() != 4 or aux_slab.shape[1] not in (SAFARA_AUX_BT, SAFARA_AUX_SP):
+        raise ValueError(f"aux_slab must be (nzl, 6|7, ny, sy), got {tuple(aux_slab.shape)}")
+    _check_shape(aux_slab, (nzl, aux_slab.shape[1], ny, pitch(nx)), "aux_slab")
     dims = canonical_dims(nx, ny, nz)
     flags = SAFARA_FLAG_STRICT if strict else 0
     check(lib().safara_rhs_slab_aux(u_slab.data_ptr(), forcing_slab.data_ptr(),
@@ -231,7 +362,19 @@ def rhs_slab_aux(u_slab, forcing_slab, out_slab, aux_slab, nx: int, nz: int, k0:
     return aux_slab
 
 
-_norm_work: dict[int, torch.Tensor] = {}
+# scratch of safara_norm_work_doubles() doubles, one per (device, stream): two
+# reductions on different streams never share partials
+_norm_work: dict[tuple[int, int], torch.Tensor] = {}
+
+
+def _work_for(r: torch.Tensor, stream) -> torch.Tensor:
+    dev = r.device.index if r.device.index is not None else torch.cuda.current_device()
+    key = (dev, int(_stream_ptr(stream) or 0))
+    work = _norm_work.get(key)
+    if work is None:
+        work = torch.empty(lib().safara_norm_work_doubles(), dtype=torch.float64, device=r.device)
+        _norm_work[key] = work
+    return work
 
 
 def rhs_sumsq(r: torch.Tensor, nx: int, nz: int | None = None, k0: int = 0, stream=None,
@@ -239,15 +382,14 @@ def rhs_sumsq(r: torch.Tensor, nx: int, nz: int | None = None, k0: int = 0, stre
     """Per-component sums of rhs^2 over the interior points of the planes
     ``r`` holds (plane p = global k0+p); a 5-element device tensor (async)."""
     _check_field(r, "rhs")
-    nzl, _, ny, _ = r.shape
+    nzl = r.shape[0]
     nz = nzl if nz is None else nz
     if dims is None:
+        _, ny = _canonical_fields(nx, ((r, "rhs"), (r, "rhs")))
         dims = canonical_dims(nx, ny, nz)
-    dev = r.device.index if r.device.index is not None else torch.cuda.current_device()
-    work = _norm_work.get(dev)
-    if work is None:
-        work = torch.empty(lib().safara_norm_work_doubles(), dtype=torch.float64, device=r.device)
-        _norm_work[dev] = work
+    else:
+        _check_numel(r, dims, nzl, "rhs")
+    work = _work_for(r, stream)
     if out is None:
         out = torch.empty(5, dtype=torch.float64, device=r.device)
     check(lib().safara_rhs_sumsq(r.data_ptr(), ctypes.byref(dims), int(k0), int(nzl),
@@ -256,12 +398,25 @@ def rhs_sumsq(r: torch.Tensor, nx: int, nz: int | None = None, k0: int = 0, stre
     return out
 
 
+def rhs_rms(r: torch.Tensor, nx: int, stream=None, out: torch.Tensor | None = None) -> torch.Tensor:
+    """NPB rhs_norm of a full-grid canonical rhs, computed entirely on the
+    device (safara_rhs_rms): a 5-element device tensor sqrt(sum rhs(m)^2 /
+    ((nx-2)(ny-2)(nz-2))) (async)."""
+    _check_field(r, "rhs")
+    nz, ny = _canonical_fields(nx, ((r, "rhs"), (r, "rhs")))
+    dims = canonical_dims(nx, ny, nz)
+    work = _work_for(r, stream)
+    if out is None:
+        out = torch.empty(5, dtype=torch.float64, device=r.device)
+    check(lib().safara_rhs_rms(r.data_ptr(), ctypes.byref(dims), work.data_ptr(), out.data_ptr(),
+                               _stream_ptr(stream)), "safara_rhs_rms")
+    return out
+
+
 def rhs_norm(r: torch.Tensor, nx: int, stream=None) -> np.ndarray:
-    """NPB rhs_norm of a full-grid canonical rhs: sqrt(sum rhs(m)^2 /
-    ((nx-2)(ny-2)(nz-2))) per component (host numpy, synchronises)."""
-    nz, _, ny, _ = r.shape
-    s = rhs_sumsq(r, nx, stream=stream).cpu().numpy()
-    return np.sqrt(s / ((nx - 2) * (ny - 2) * (nz - 2)))
+    """NPB rhs_norm of a full-grid canonical rhs as a host numpy array
+    (safara_rhs_rms, then a device->host copy: synchronises)."""
+    return rhs_rms(r, nx, stream=stream).cpu().numpy()
 
 
 # ---- SURVEY §8(f) f4(i): the 355.seismic dz loop (PAPER.md Fig. 8) --------

@@ -1,0 +1,257 @@
+"""GPU tests of the boundary's named entry points:
+``safara_rhs`` itself (the north_star call, canonical layout, production),
+the sharded pass on a library-owned NCCL communicator
+(``safara_shard_init`` / ``safara_rhs_sharded(_ex)`` / ``safara_shard_rms``
+/ ``safara_shard_finalize``) at nranks = 1 and, where the box has two GPUs,
+2 ranks over NCCL, and the device-side NPB rhs_norm (``safara_rhs_rms``).
+Bars: STRICT bit-identical to the oracle; production within reading c5."""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+
+import nasgen
+import oracle
+import paper_conf_icpp_tiankexc16_b200 as sr
+from paper_conf_icpp_tiankexc16_b200 import _abi
+from paper_conf_icpp_tiankexc16_b200 import dist as sd
+
+pytestmark = pytest.mark.gpu
+
+RTOL, ATOL = 1e-12, 1e-14
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _init():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    sr.init(0)
+
+
+def assert_tol(g, o):
+    err = np.abs(g - o)
+    bound = RTOL * np.abs(o) + ATOL
+    assert (err <= bound).all(), f"worst ratio {(err / bound).max():.3g}"
+
+
+@pytest.mark.parametrize("bench,cls", [("BT", "S"), ("BT", "C")])
+def test_safara_rhs_entry_point(bench, cls):
+    """safara_rhs(u, forcing, rhs, nx, ny, nz, coeffs, stream) -- no flags,
+    canonical layout -- is the production variant: bit-identical to
+    safara_rhs_ex(flags=0) and within c5 of the oracle; STRICT through _ex
+    is bit-identical to the oracle on the same inputs."""
+    import ctypes
+    inp = nasgen.make_class(bench, cls, seed=2, B=1e-2)
+    nz, ny, nx, _ = inp.u.shape
+    c = sr.coeffs_nas(nx, ny, nz, inp.dt)
+    du, df = sr.pack(inp.u), sr.pack(inp.forcing)
+    r1 = torch.full_like(du, float("nan"))
+    r2 = torch.full_like(du, float("nan"))
+    r3 = torch.full_like(du, float("nan"))
+    L = _abi.lib()
+    n0 = sr.launch_count()
+    _abi.check(L.safara_rhs(du.data_ptr(), df.data_ptr(), r1.data_ptr(), nx, ny, nz,
+                            ctypes.byref(c), torch.cuda.current_stream().cuda_stream),
+               "safara_rhs")
+    d = sr.canonical_dims(nx, ny, nz)
+    _abi.check(L.safara_rhs_ex(du.data_ptr(), df.data_ptr(), r2.data_ptr(), ctypes.byref(d),
+                               ctypes.byref(c), 0, torch.cuda.current_stream().cuda_stream),
+               "safara_rhs_ex")
+    sr.rhs(du, df, r3, nx, c, strict=True)
+    torch.cuda.synchronize()
+    assert sr.launch_count() == n0 + 3
+    # (pitch padding columns stay NaN: compare the grid points)
+    assert np.array_equal(sr.unpack(r1, nx), sr.unpack(r2, nx))
+    o = oracle.compute_rhs(inp.u, inp.forcing, dt=inp.dt, threads=8)
+    assert_tol(sr.unpack(r1, nx), o)
+    assert np.array_equal(sr.unpack(r3, nx), o)
+
+
+def test_binding_rhs_calls_safara_rhs():
+    """The binding's canonical production call routes to safara_rhs (same
+    bits as the direct call above; shape errors raise before the C side)."""
+    inp = nasgen.make_class("BT", "S", seed=3)
+    nz, ny, nx, _ = inp.u.shape
+    c = sr.coeffs_nas(nx, ny, nz, inp.dt)
+    du, df = sr.pack(inp.u), sr.pack(inp.forcing)
+    r = torch.empty_like(du)
+    sr.rhs(du, df, r, nx, c)
+    torch.cuda.synchronize()
+    assert_tol(sr.unpack(r, nx), oracle.compute_rhs(inp.u, inp.forcing, dt=inp.dt))
+    with pytest.raises(ValueError):
+        sr.rhs(du, df[:-1].contiguous(), r, nx, c)          # forcing one plane short
+    with pytest.raises(ValueError):
+        sr.rhs(du, df, r, nx + 8, c)                         # pitch(nx) mismatch
+    with pytest.raises(ValueError):
+        sr.rhs_slab(du, df, r, nx, nz, 0, c)                 # u without ghost planes
+
+
+def _shard1():
+    return sr.shard_init(sr.get_unique_id(), 0, 1, torch.cuda.current_device())
+
+
+@pytest.mark.parametrize("strict", [True, False])
+def test_sharded_nranks1_vs_oracle(strict):
+    """nranks = 1: the sharded call is one PART_ALL slab pass."""
+    inp = nasgen.make_class("BT", "W", seed=1, B=1e-2)
+    nz, ny, nx, _ = inp.u.shape
+    c = sr.coeffs_nas(nx, ny, nz, inp.dt)
+    s = sd.make_slab(sr.pack(inp.u, device="cpu"), sr.pack(inp.forcing, device="cpu"), nx, 0, 1,
+                     device="cuda")
+    s.rhs.fill_(float("nan"))
+    h = _shard1()
+    try:
+        assert sr.shard_rank(h) == (0, 1)
+        n0 = sr.launch_count()
+        sr.rhs_sharded(h, s.u, s.forcing, s.rhs, nx, nz, 0, c, strict=strict)
+        rms = sr.shard_rms(h, s.rhs, nx, nz, 0)
+        torch.cuda.synchronize()
+        assert sr.launch_count() == n0 + 1 + 3       # PART_ALL; sumsq (2) + finish
+    finally:
+        sr.shard_finalize(h)
+    o = oracle.compute_rhs(inp.u, inp.forcing, dt=inp.dt)
+    g = sr.unpack(s.rhs, nx)
+    if strict:
+        assert np.array_equal(g, o)
+    else:
+        assert_tol(g, o)
+    want = np.sqrt(oracle.rhs_sumsq(g) / ((nx - 2) * (ny - 2) * (nz - 2)))
+    np.testing.assert_allclose(rms.cpu().numpy(), want, rtol=1e-13, atol=0)
+
+
+def test_sharded_argument_checks_on_device():
+    inp = nasgen.make_class("BT", "S", seed=1)
+    nz, ny, nx, _ = inp.u.shape
+    c = sr.coeffs_nas(nx, ny, nz, inp.dt)
+    h = _shard1()
+    try:
+        s = sd.make_slab(sr.pack(inp.u, device="cpu"), sr.pack(inp.forcing, device="cpu"), nx,
+                         0, 1, device="cuda")
+        # a 1-rank shard must own the whole grid: k0 = 0 and k0 + nzl = nz
+        f2 = s.forcing[: nz - 2].contiguous()
+        r2 = torch.empty_like(f2)
+        u2 = s.u[: nz + 2].contiguous()
+        with pytest.raises(sr.SafaraError) as e:
+            sr.rhs_sharded(h, u2, f2, r2, nx, nz, 0, c)
+        assert e.value.code == -2
+    finally:
+        sr.shard_finalize(h)
+
+
+def test_rhs_rms_device_norm():
+    """safara_rhs_rms: NPB rhs_norm finished on the device == oracle sums."""
+    inp = nasgen.make_class("SP", "W", seed=1, B=1e-2)
+    nz, ny, nx, _ = inp.u.shape
+    c = sr.coeffs_nas(nx, ny, nz, inp.dt)
+    du, df = sr.pack(inp.u), sr.pack(inp.forcing)
+    r = torch.empty_like(du)
+    sr.rhs(du, df, r, nx, c, strict=True)
+    rms = sr.rhs_rms(r, nx)
+    torch.cuda.synchronize()
+    o = oracle.compute_rhs(inp.u, inp.forcing, dt=inp.dt)
+    want = np.sqrt(oracle.rhs_sumsq(o) / ((nx - 2) * (ny - 2) * (nz - 2)))
+    np.testing.assert_allclose(rms.cpu().numpy(), want, rtol=1e-13, atol=0)
+    np.testing.assert_allclose(sr.rhs_norm(r, nx), want, rtol=1e-13, atol=0)
+
+
+def test_peer_halo_fails_clearly_under_expandable_segments():
+    """CUDA IPC cannot export VMM (expandable-segment) allocations; PeerHalo
+    must raise PeerHaloUnavailable on every rank (not hang, not run), and the
+    NCCL path (NcclShard) is the fallback the bench takes."""
+    import torch.distributed as dist
+    alloc = torch.cuda.memory
+    alloc._set_allocator_settings("expandable_segments:True")
+    try:
+        t = torch.empty(64 << 20, dtype=torch.uint8, device="cuda")   # a new (VMM) segment
+        try:
+            sr.ipc_get(t)
+            exported = True
+        except sr.SafaraError as e:
+            exported = False
+            assert e.code == -7
+        if exported:
+            pytest.skip("this allocator still returned an IPC-exportable block")
+        s = socket.socket()
+        s.bind(("127.0.0.1", 0))
+        port = s.getsockname()[1]
+        s.close()
+        os.environ["MASTER_ADDR"] = "127.0.0.1"
+        os.environ["MASTER_PORT"] = str(port)
+        dist.init_process_group("gloo", rank=0, world_size=1)
+        try:
+            inp = nasgen.make_class("BT", "S", seed=1)
+            nz, ny, nx, _ = inp.u.shape
+            slab = sd.make_slab(sr.pack(inp.u, device="cpu"), sr.pack(inp.forcing, device="cpu"),
+                                nx, 0, 1, device="cuda")
+            with pytest.raises(sd.PeerHaloUnavailable):
+                sd.PeerHalo(slab)
+            # the fallback: the library's NCCL shard on the same (VMM) buffers
+            sh = sd.NcclShard(0, 1, torch.cuda.current_device())
+            try:
+                c = sr.coeffs_nas(nx, ny, nz, inp.dt)
+                sd.rhs_sharded(slab, c, sh, strict=True)
+                torch.cuda.synchronize()
+            finally:
+                sh.close()
+            assert np.array_equal(sr.unpack(slab.rhs, nx),
+                                  oracle.compute_rhs(inp.u, inp.forcing, dt=inp.dt))
+        finally:
+            dist.destroy_process_group()
+    finally:
+        alloc._set_allocator_settings("expandable_segments:False")
+
+
+def _nccl_worker(rank, world, port, q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    import torch.distributed as dist
+    torch.cuda.set_device(rank)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        inp = nasgen.make_class("BT", "A", seed=1, B=1e-2)
+        nz, ny, nx, _ = inp.u.shape
+        ug, fg = sr.pack(inp.u, device="cpu"), sr.pack(inp.forcing, device="cpu")
+        s = sd.make_slab(ug, fg, nx, rank, world, device=f"cuda:{rank}")
+        s.u[: sd.GHOST] = float("nan")           # ghosts must come from the exchange
+        s.u[-sd.GHOST:] = float("nan")
+        c = sr.coeffs_nas(nx, ny, nz, inp.dt)
+        sh = sd.NcclShard(rank, world, rank)
+        try:
+            for _ in range(3):
+                sd.rhs_sharded(s, c, sh, strict=True)
+            rms = sh.rms(s)
+            torch.cuda.synchronize()
+        finally:
+            sh.close()
+        q.put((rank, s.k0, sr.unpack(s.rhs, nx), rms.cpu().numpy()))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.skipif(not torch.cuda.is_available() or torch.cuda.device_count() < 2,
+                    reason="needs 2 GPUs")
+def test_sharded_two_ranks_nccl():
+    import torch.multiprocessing as mp
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    procs = [ctx.Process(target=_nccl_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    got = sorted((q.get(timeout=300) for _ in range(2)), key=lambda x: x[0])
+    for p in procs:
+        p.join(timeout=120)
+        assert p.exitcode == 0
+    inp = nasgen.make_class("BT", "A", seed=1, B=1e-2)
+    o = oracle.compute_rhs(inp.u, inp.forcing, dt=inp.dt)
+    g = np.concatenate([x[2] for x in got], axis=0)
+    assert np.array_equal(g, o)
+    n = inp.u.shape[0]
+    want = np.sqrt(oracle.rhs_sumsq(o) / (n - 2) ** 3)
+    for x in got:
+        np.testing.assert_allclose(x[3], want, rtol=1e-13, atol=0)
