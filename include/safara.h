@@ -365,6 +365,55 @@ int safara_seismic_dz(const double *vz1, const double *vz2, const double *vz3,
                       double *value_dz, const safara_dims3_t *dims, double h,
                       void *stream);
 
+/* ---- a whole NPB BT time step on the GPU -----------
+ *
+ * NPB BT's ADI step (adi.f: compute_rhs; x_solve; y_solve; z_solve; add) on
+ * canonical device arrays, so that the library reproduces NPB's own
+ * verification norms (tests/golden/npb_bt_verify.txt; the paper runs NPB-ACC
+ * BT).  The solves are NPB's approximate-factorisation
+ * line solves: along every interior grid line of a direction the 5x5
+ * block-tridiagonal system (flux Jacobian fjac, viscous Jacobian njac,
+ * dx/dy/dz diagonal, identity end blocks) by block Gaussian elimination
+ * without pivoting and back substitution, in place on rhs; NPB operation
+ * order without FMA contraction (bit-identical to the oracle on bit-identical
+ * inputs).  Not the hot path: one thread per line.
+ *   safara_bt_coeffs_t / safara_bt_coeffs_nas: the set_constants values the
+ *       solves use (host).  SAFARA_ERR_ARG / SAFARA_ERR_SHAPE (extent < 2).
+ *   safara_bt_work_doubles: device scratch (doubles) the solves need:
+ *       25 x max over directions of (lines x points per line); < 0 = error.
+ *   safara_bt_solve: dir 0 = x_solve, 1 = y_solve, 2 = z_solve of rhs in
+ *       place.  u, rhs: canonical [k][m][j][i] (dims: sm >= sy*ny,
+ *       sk >= 5*sm, else SAFARA_ERR_LAYOUT), aux: the BT aux fields of u
+ *       (safara_rhs_aux, naux = 6, plane stride 6*sm), work: scratch.  One
+ *       launch.  Errors: SAFARA_ERR_ARG (NULL, overlap, dir), descriptor
+ *       errors, SAFARA_ERR_ALIGN (8 B), SAFARA_ERR_CUDA.
+ *   safara_bt_add: u += rhs at the interior points (add.f).  One launch.
+ *   safara_bt_step: safara_rhs_aux (flags: SAFARA_FLAG_STRICT selects the
+ *       bit-identical rhs/aux variant), the three solves, add: 5 launches,
+ *       asynchronous, u updated in place, rhs/aux/work overwritten.
+ *   safara_error_norm: NPB error_norm into 5 device doubles: sqrt(sum over
+ *       ALL points of (u - u_exact)^2 / (nx-2) / (ny-2) / (nz-2)); work of
+ *       safara_norm_work_doubles(); deterministic; 2 launches.             */
+typedef struct {
+    double dt, c1, c2, c3c4, c1c5, con43;
+    double tx1, tx2, ty1, ty2, tz1, tz2;
+    double dx[5], dy[5], dz[5];
+} safara_bt_coeffs_t;
+int safara_bt_coeffs_nas(int nx, int ny, int nz, double dt, safara_bt_coeffs_t *out);
+int safara_bt_work_doubles(int nx, int ny, int nz);
+int safara_bt_solve(int dir, const double *u, const double *aux, double *rhs,
+                    double *work, const safara_dims_t *dims,
+                    const safara_bt_coeffs_t *bc, void *stream);
+int safara_bt_add(double *u, const double *rhs, const safara_dims_t *dims,
+                  void *stream);
+int safara_bt_step(double *u, const double *forcing, double *rhs, double *aux,
+                   double *work, const safara_dims_t *dims,
+                   const safara_coeffs_t *coeffs, const safara_bt_coeffs_t *bc,
+                   int flags, void *stream);
+int safara_error_norm(const double *u, const double *u_exact,
+                      const safara_dims_t *dims, double *work, double *rms,
+                      void *stream);
+
 /* End-to-end call with HOST arrays (canonical layout): copies u and forcing
  * host->device into the caller's device buffers u_dev/forcing_dev, runs the
  * pass into rhs_dev and copies rhs device->host.  The grid is cut into

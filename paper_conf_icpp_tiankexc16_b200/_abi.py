@@ -37,6 +37,13 @@ class Coeffs(ctypes.Structure):
         (n, ctypes.c_double * 5) for n in ("dxt", "dyt", "dzt", "xxcon", "yycon", "zzcon")]
 
 
+class BtCoeffs(ctypes.Structure):
+    """safara_bt_coeffs_t."""
+    _fields_ = [(n, ctypes.c_double) for n in
+                ("dt", "c1", "c2", "c3c4", "c1c5", "con43", "tx1", "tx2", "ty1", "ty2", "tz1",
+                 "tz2")] + [(n, ctypes.c_double * 5) for n in ("dx", "dy", "dz")]
+
+
 class Dims3(ctypes.Structure):
     """safara_dims3_t: the shared 3-D descriptor of the seismic dz loop."""
     _fields_ = [(n, ctypes.c_int32) for n in ("nx", "ny", "nz", "sy", "sk")]
@@ -111,6 +118,15 @@ _SIGS = {
     "safara_shard_rank": ([_dp, ctypes.POINTER(ctypes.c_int), ctypes.POINTER(ctypes.c_int)],
                           ctypes.c_int),
     "safara_shard_finalize": ([_dp], ctypes.c_int),
+    "safara_bt_coeffs_nas": ([ctypes.c_int] * 3 + [ctypes.c_double, ctypes.POINTER(BtCoeffs)],
+                             ctypes.c_int),
+    "safara_bt_work_doubles": ([ctypes.c_int] * 3, ctypes.c_int),
+    "safara_bt_solve": ([ctypes.c_int, _dp, _dp, _dp, _dp, ctypes.POINTER(Dims),
+                         ctypes.POINTER(BtCoeffs), _dp], ctypes.c_int),
+    "safara_bt_add": ([_dp, _dp, ctypes.POINTER(Dims), _dp], ctypes.c_int),
+    "safara_bt_step": ([_dp] * 5 + [ctypes.POINTER(Dims), ctypes.POINTER(Coeffs),
+                                    ctypes.POINTER(BtCoeffs), ctypes.c_int, _dp], ctypes.c_int),
+    "safara_error_norm": ([_dp, _dp, ctypes.POINTER(Dims), _dp, _dp, _dp], ctypes.c_int),
     "safara_launch_count": ([], ctypes.c_int64),
     "safara_kernel_info": ([ctypes.c_int, ctypes.POINTER(KernelInfo)], ctypes.c_int),
     "safara_strerror": ([ctypes.c_int], ctypes.c_char_p),

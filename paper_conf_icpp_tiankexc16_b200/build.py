@@ -46,6 +46,7 @@ UNITS = [
     ("seismic.cu", ["-Xptxas", "-v"]),
     ("api.cu", []),
     ("shard.cu", ["-I" + _nccl_include()]),
+    ("bt_solve.cu", ["--fmad=false", "-Xptxas", "-v"]),
 ]
 DEPS = ["rhs_kernel.cuh", "rhs_variant.inc", "safara_internal.h"]
 

@@ -120,6 +120,17 @@ cudaError_t launch_seismic_dz(const double *vz1, const double *vz2, const double
                               int nx, int ny, int nz, int sy, int sk, double h, int sms,
                               cudaStream_t s);
 
+// bt_solve.cu: SURVEY §8(f) f4(ii), the NPB BT line solves / add / error norm
+int bt_work_doubles(int nx, int ny, int nz);
+cudaError_t launch_bt_solve(int dir, const double *u, const double *aux, double *rhs,
+                            double *work, int nx, int ny, int nz, int sy, int sm, int sk, int ska,
+                            const safara_bt_coeffs_t &bc, cudaStream_t s);
+cudaError_t launch_bt_add(double *u, const double *rhs, int nx, int ny, int nz, int sy, int sm,
+                          int sk, int sms, cudaStream_t s);
+int err_norm_grid();
+cudaError_t launch_error_norm(const double *u, const double *ue, int nx, int ny, int nz, int sy,
+                              int sm, int sk, double *work, double *rms, cudaStream_t s);
+
 // attr: 4 entries (production NAS path, general coefficients, aux, NAS + aux)
 cudaError_t setup_rhs_fast(int *ctas_per_sm, cudaFuncAttributes *attr);
 cudaError_t setup_rhs_strict(int *ctas_per_sm, cudaFuncAttributes *attr);

@@ -14,8 +14,8 @@ import numpy as np
 import torch
 
 from ._abi import (SAFARA_AUX_BT, SAFARA_AUX_SP, SAFARA_FLAG_STRICT, SAFARA_IPC_HANDLE_BYTES,
-                   SAFARA_PART_ALL, SAFARA_UNIQUE_ID_BYTES, Coeffs, Dims, Dims3, KernelInfo, Peer,
-                   check, lib)
+                   SAFARA_PART_ALL, SAFARA_UNIQUE_ID_BYTES, BtCoeffs, Coeffs, Dims, Dims3,
+                   KernelInfo, Peer, check, lib)
 
 _initialised: set[int] = set()
 
@@ -436,3 +436,61 @@ def seismic_dz(vz1: torch.Tensor, vz2: torch.Tensor, vz3: torch.Tensor, out: tor
                                   ctypes.byref(d), float(h), _stream_ptr(stream)),
           "safara_seismic_dz")
     return out
+
+
+# ---- a whole NPB BT time step ---------------------------
+
+def bt_coeffs_nas(nx: int, ny: int, nz: int, dt: float) -> BtCoeffs:
+    c = BtCoeffs()
+    check(lib().safara_bt_coeffs_nas(nx, ny, nz, float(dt), ctypes.byref(c)),
+          "safara_bt_coeffs_nas")
+    return c
+
+
+class BtState:
+    """Device state of an NPB BT run on canonical tensors: u (updated in
+    place), forcing, and the rhs / aux / solver scratch the step overwrites."""
+
+    def __init__(self, u: torch.Tensor, forcing: torch.Tensor, nx: int, dt: float):
+        _check_field(u, "u")
+        _check_field(forcing, "forcing")
+        nz, ny = _canonical_fields(nx, ((u, "u"), (forcing, "forcing"), (forcing, "forcing")))
+        self.nx, self.ny, self.nz, self.dt = nx, ny, nz, dt
+        self.u, self.forcing = u, forcing
+        self.rhs = torch.empty_like(u)
+        self.aux = torch.empty((nz, SAFARA_AUX_BT, ny, pitch(nx)), dtype=torch.float64,
+                               device=u.device)
+        w = lib().safara_bt_work_doubles(nx, ny, nz)
+        check(min(w, 0), "safara_bt_work_doubles")
+        self.work = torch.empty(w, dtype=torch.float64, device=u.device)
+        self.dims = canonical_dims(nx, ny, nz)
+        self.coeffs = coeffs_nas(nx, ny, nz, dt)
+        self.bt = bt_coeffs_nas(nx, ny, nz, dt)
+
+    def step(self, strict: bool = False, stream=None):
+        """One ADI step: safara_bt_step (rhs_aux, x/y/z_solve, add; 5 launches)."""
+        check(lib().safara_bt_step(self.u.data_ptr(), self.forcing.data_ptr(),
+                                   self.rhs.data_ptr(), self.aux.data_ptr(), self.work.data_ptr(),
+                                   ctypes.byref(self.dims), ctypes.byref(self.coeffs),
+                                   ctypes.byref(self.bt), SAFARA_FLAG_STRICT if strict else 0,
+                                   _stream_ptr(stream)), "safara_bt_step")
+
+    def solve(self, direction: int, stream=None):
+        """One line solve of self.rhs in place (aux must hold u's fields)."""
+        check(lib().safara_bt_solve(int(direction), self.u.data_ptr(), self.aux.data_ptr(),
+                                    self.rhs.data_ptr(), self.work.data_ptr(),
+                                    ctypes.byref(self.dims), ctypes.byref(self.bt),
+                                    _stream_ptr(stream)), "safara_bt_solve")
+
+    def verify_norms(self, u_exact: torch.Tensor, strict: bool = False, stream=None):
+        """NPB BT verify on the device: (xce, xcr) as 5-element device tensors,
+        xce = error_norm(u, u_exact), xcr = rhs_norm(compute_rhs(u)) / dt."""
+        _check_shape(u_exact, tuple(self.u.shape), "u_exact")
+        work = _work_for(self.u, stream)
+        xce = torch.empty(5, dtype=torch.float64, device=self.u.device)
+        check(lib().safara_error_norm(self.u.data_ptr(), u_exact.data_ptr(),
+                                      ctypes.byref(self.dims), work.data_ptr(), xce.data_ptr(),
+                                      _stream_ptr(stream)), "safara_error_norm")
+        rhs(self.u, self.forcing, self.rhs, self.nx, self.coeffs, strict=strict, stream=stream)
+        xcr = rhs_rms(self.rhs, self.nx, stream=stream)
+        return xce, xcr / self.dt
