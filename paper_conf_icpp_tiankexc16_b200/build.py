@@ -48,7 +48,7 @@ UNITS = [
     ("shard.cu", ["-I" + _nccl_include()]),
     ("bt_solve.cu", ["--fmad=false", "-Xptxas", "-v"]),
 ]
-DEPS = ["rhs_kernel.cuh", "rhs_variant.inc", "safara_internal.h"]
+DEPS = ["rhs_kernel.cuh", "rhs_ws.cuh", "rhs_variant.inc", "safara_internal.h"]
 
 
 def _mtime(p):
@@ -56,9 +56,11 @@ def _mtime(p):
 
 
 def build(force: bool = False, verbose: bool = False, extra: list[str] | None = None,
-          out: str | None = None) -> str:
-    """Compile (if stale) and return the path of libsafara_rhs.so (or ``out``)."""
-    os.makedirs(BUILD, exist_ok=True)
+          out: str | None = None, objdir: str | None = None) -> str:
+    """Compile (if stale) and return the path of libsafara_rhs.so (or ``out``;
+    ``objdir`` keeps a variant build's objects apart from the default ones)."""
+    objdir = objdir or BUILD
+    os.makedirs(objdir, exist_ok=True)
     lib = out or LIB
     extra = list(extra or [])
     srcs = [os.path.join(CSRC, u) for u, _ in UNITS] + [os.path.join(CSRC, d) for d in DEPS]
@@ -69,7 +71,7 @@ def build(force: bool = False, verbose: bool = False, extra: list[str] | None = 
     objs = []
     ptxas_log = []
     for unit, flags in UNITS:
-        obj = os.path.join(BUILD, unit.replace(".cu", ".o"))
+        obj = os.path.join(objdir, unit.replace(".cu", ".o"))
         cmd = [NVCC, *COMMON, *flags, *extra, "-c", os.path.join(CSRC, unit), "-o", obj]
         res = subprocess.run(cmd, capture_output=True, text=True)
         if res.returncode != 0:

@@ -35,6 +35,7 @@ struct DeviceState {
     int sms = 0;
     int ctas_fast = 0, ctas_strict = 0;
     cudaFuncAttributes attr_fast[4]{}, attr_strict[4]{};
+    cudaFuncAttributes attr_ws_fast[2]{}, attr_ws_strict[2]{};
     // copy engines for safara_rhs_host's H2D / D2H pipeline (created at init)
     cudaStream_t h2d = nullptr, d2h = nullptr;
     cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
@@ -59,6 +60,7 @@ struct Tune {
     int split_bias = 0;  // experiments: shift the lockstep k-split points (no peer)
     int peer_bias_maxpart = 6;  // peer_bias only for k-parts of at most this many planes
     int peer_timeout_ms = 30000;  // f2 flag waits: give up and trap after this long
+    int ws = 0;  // 1: warp-specialised kernel (rhs_ws.cuh) where it applies (A/B: 1-2 % slower, off)
 } g_tune;
 
 int env_int(const char *name, int dflt) {
@@ -339,8 +341,17 @@ int launch(const double *u, const double *f, double *r, const safara_dims_t &d, 
     bool ud = true;
     for (int ax = 0; ax < 3; ++ax)
         for (int m = 1; m < 5; ++m) ud = ud && (p.c.d1[ax][m] == p.c.d1[ax][0]);
-    cudaError_t e = strict ? launch_rhs_strict(umap, fmap, p, ud, stream)
-                           : launch_rhs_fast(umap, fmap, p, ud, stream);
+    // the warp-specialised kernel serves launches whose CTAs each own one
+    // (column tile, k range) segment: lockstep over a single plane range,
+    // without the f1 aux output or the f2 peer halo
+    const bool ws = g_tune.ws && lockstep && p.parts > 0 && p.n0 == p.nplanes && !aux && !peer;
+    cudaError_t e;
+    if (ws)
+        e = strict ? launch_rhs_ws_strict(umap, fmap, p, ud, stream)
+                   : launch_rhs_ws_fast(umap, fmap, p, ud, stream);
+    else
+        e = strict ? launch_rhs_strict(umap, fmap, p, ud, stream)
+                   : launch_rhs_fast(umap, fmap, p, ud, stream);
     if (e != cudaSuccess) return SAFARA_ERR_CUDA;
     g_launches.fetch_add(1, std::memory_order_relaxed);
     return SAFARA_OK;
@@ -434,6 +445,7 @@ int safara_rhs_init(int device) {
     g_tune.split_bias = env_int("SAFARA_SPLIT_BIAS", g_tune.split_bias);
     g_tune.peer_bias_maxpart = env_int("SAFARA_PEER_BIAS_MAXPART", g_tune.peer_bias_maxpart);
     g_tune.peer_timeout_ms = std::max(1, env_int("SAFARA_PEER_TIMEOUT_MS", g_tune.peer_timeout_ms));
+    g_tune.ws = env_int("SAFARA_WS", g_tune.ws);
     int major = 0, minor = 0, sms = 0;
     if (cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, device) ||
         cudaDeviceGetAttribute(&minor, cudaDevAttrComputeCapabilityMinor, device) ||
@@ -456,6 +468,8 @@ int safara_rhs_init(int device) {
     st.sms = sms;
     cudaError_t e = setup_rhs_fast(&st.ctas_fast, st.attr_fast);
     if (e == cudaSuccess) e = setup_rhs_strict(&st.ctas_strict, st.attr_strict);
+    if (e == cudaSuccess) e = setup_rhs_ws_fast(st.attr_ws_fast);
+    if (e == cudaSuccess) e = setup_rhs_ws_strict(st.attr_ws_strict);
     if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&st.h2d, cudaStreamNonBlocking);
     if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&st.d2h, cudaStreamNonBlocking);
     if (e == cudaSuccess) e = cudaEventCreateWithFlags(&st.ev_fork, cudaEventDisableTiming);

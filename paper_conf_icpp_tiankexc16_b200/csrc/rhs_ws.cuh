@@ -1,0 +1,428 @@
+// rhs_ws.cuh -- warp-specialised variant of the compute_rhs pass (round 2).
+//
+// Same arithmetic and the same per-thread k march as rhs_kernel.cuh (one
+// thread per (i,j) column, register window along k = SAFARA's
+// inter-iteration scalar replacement, Fig. 6),
+// but the CTA is split into two roles:
+//
+//  * 4 PRODUCER warps (one warpgroup, registers handed to the consumers with
+//    setmaxnreg.dec): one lane issues the TMA loads of the u / forcing plane
+//    tiles into the STAGES-deep ring when the consumers release a slot
+//    (mbarrier `empty`, no atomics); then all 128 producer threads evaluate
+//    the step-0 fields rho_i = 1/u1 and square (App. A step 0) ONCE for every
+//    point of the plane tile plus a halo of one, into an aux ring in shared
+//    memory, and signal `afull`.
+//  * TY CONSUMER warps (setmaxnreg.inc), one tile row each: every neighbour's
+//    rho_i / square now comes from that aux tile (one 16-byte load) instead of
+//    being recomputed per use (round 1 evaluated aux_of four times per point:
+//    own, the xi tile-edge lanes, both eta rows) or shuffled; the own values
+//    of plane k+1 are loaded, not computed.
+//
+// SAFARA's cost model (L x C) placed the values
+// with reuse > 1 that other threads need in shared memory; the aux fields have
+// reuse 5 (own + 4 in-plane neighbours) and were recomputed in round 1 only
+// because a consumer-side producer needed cross-warp waits.  A producer
+// warpgroup working ahead of the consumers removes those waits.
+//
+// Scope: launches whose CTAs each own ONE (column tile, k range) segment
+// (the lockstep schedule) without the f1 aux output or the f2 peer halo;
+// everything else runs rhs_kernel.cuh (launch() decides).
+#pragma once
+
+namespace safara {
+namespace dev {
+
+constexpr int WS_PW = 4;                     // producer warps (one warpgroup)
+constexpr int WS_THREADS = (TY + WS_PW) * 32;
+constexpr int AXW = TX + 2, AYW = TY + 2;    // aux tile: columns i0-1..i0+TX, rows j0-1..j0+TY
+constexpr int A_SLOT = AXW * AYW;            // double2 per aux slot
+#ifndef SAFARA_WS_SLEEP
+#define SAFARA_WS_SLEEP 20000   // producer waits: suspend-time hint (ns), 0 = plain try_wait
+#endif
+__device__ __forceinline__ void ws_pwait(uint64_t *bar, uint32_t parity) {
+#if SAFARA_WS_SLEEP > 0
+    mbar_wait_sleep(bar, parity, SAFARA_WS_SLEEP);
+#else
+    mbar_wait(bar, parity);
+#endif
+}
+#ifndef SAFARA_WS_PREG
+#define SAFARA_WS_PREG 32                    // producer registers after setmaxnreg.dec
+#endif
+// consumer registers after setmaxnreg.inc: the rest of the 64K register file
+constexpr int WS_CREG = ((65536 / 32 - WS_PW * SAFARA_WS_PREG) / TY) / 8 * 8;
+static_assert(WS_CREG >= 128 && WS_CREG <= 256, "consumer register budget");
+
+// Shared memory: a u ring of WS_US plane tiles (with halo 2), the aux ring
+// (one (rho_i, square) tile per u slot) and a separate, shallower forcing ring
+// of WS_FS slots -- forcing(k) is read only at step k, u(k) already at step
+// k-2 (own column), so splitting the rings buys one more u plane of TMA
+// lookahead in the same shared memory.
+#ifndef SAFARA_WS_US
+#define SAFARA_WS_US 5
+#endif
+#ifndef SAFARA_WS_FS
+#define SAFARA_WS_FS 3
+#endif
+constexpr int WS_US = SAFARA_WS_US, WS_FS = SAFARA_WS_FS;
+constexpr size_t WS_U_BYTES = (size_t)WS_US * U_SLOT * 8;
+// (padded: the forcing ring behind it is a TMA destination, 128-byte aligned)
+constexpr size_t WS_AUX_BYTES = ((size_t)WS_US * A_SLOT * 16 + 127) / 128 * 128;
+constexpr size_t WS_F_BYTES = (size_t)WS_FS * F_SLOT * 8;
+constexpr size_t WS_BAR_OFF = WS_U_BYTES + WS_AUX_BYTES + WS_F_BYTES;
+constexpr size_t WS_SMEM_BYTES = WS_BAR_OFF + (3 * WS_US + 2 * WS_FS) * 8;
+static_assert(WS_SMEM_BYTES <= 227 * 1024, "WS shared memory");
+static_assert(WS_U_BYTES % 128 == 0 && (U_SLOT * 8) % 128 == 0 && (F_SLOT * 8) % 128 == 0 &&
+                  (WS_U_BYTES + WS_AUX_BYTES) % 128 == 0,
+              "TMA destinations 128-byte aligned");
+
+__device__ __forceinline__ double *ws_u() { return reinterpret_cast<double *>(smem_raw); }
+__device__ __forceinline__ double2 *ws_aux() {
+    return reinterpret_cast<double2 *>(smem_raw + WS_U_BYTES);
+}
+__device__ __forceinline__ double *ws_f() {
+    return reinterpret_cast<double *>(smem_raw + WS_U_BYTES + WS_AUX_BYTES);
+}
+__device__ __forceinline__ uint64_t *ws_full() {
+    return reinterpret_cast<uint64_t *>(smem_raw + WS_BAR_OFF);
+}
+__device__ __forceinline__ uint64_t *ws_afull() { return ws_full() + WS_US; }
+__device__ __forceinline__ uint64_t *ws_empty() { return ws_full() + 2 * WS_US; }
+__device__ __forceinline__ uint64_t *ws_ffull() { return ws_full() + 3 * WS_US; }
+__device__ __forceinline__ uint64_t *ws_fempty() { return ws_ffull() + WS_FS; }
+
+// TMA of u plane k (tile with halo 2) into u slot `slot`, of forcing plane k
+// into forcing slot `slot` (coordinates as rhs_kernel.cuh issue_plane).
+__device__ __forceinline__ void ws_issue_u(const CUtensorMap *umap, const Params &P, int i0,
+                                           int j0, int k, int slot) {
+    const int kb = k - P.k0 + P.ukoff, jc = j0 - 2;
+    const int c1 = P.pos_j == 1 ? jc : (P.pos_m == 1 ? 0 : kb);
+    const int c2 = P.pos_j == 2 ? jc : (P.pos_m == 2 ? 0 : kb);
+    const int c3 = P.pos_j == 3 ? jc : (P.pos_m == 3 ? 0 : kb);
+    uint64_t *bar = &ws_full()[slot];
+    mbar_expect_tx(bar, TMA_BYTES);
+    tma_load_4d(ws_u() + (size_t)slot * U_SLOT, umap, bar, i0 - HX, c1, c2, c3);
+}
+__device__ __forceinline__ void ws_issue_f(const CUtensorMap *fmap, const Params &P, int i0,
+                                           int j0, int k, int slot) {
+    const int kf = k - P.k0;
+    const int f1 = P.pos_j == 1 ? j0 : (P.pos_m == 1 ? 0 : kf);
+    const int f2 = P.pos_j == 2 ? j0 : (P.pos_m == 2 ? 0 : kf);
+    const int f3 = P.pos_j == 3 ? j0 : (P.pos_m == 3 ? 0 : kf);
+    uint64_t *bar = &ws_ffull()[slot];
+    mbar_expect_tx(bar, TMA_BYTES_F);
+    tma_load_4d(ws_f() + (size_t)slot * F_SLOT, fmap, bar, i0 - 1, f1, f2, f3);
+}
+
+__device__ __forceinline__ void setmaxnreg_inc_consumer() {
+    asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;\n" ::"n"(WS_CREG));
+}
+__device__ __forceinline__ void setmaxnreg_dec_producer() {
+    asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;\n" ::"n"(SAFARA_WS_PREG));
+}
+
+// The CTA's segment in the lockstep schedule: column tile `col`, global
+// planes [ka, kb).
+__device__ __forceinline__ void ws_segment(const Params &P, int &col, int &ka, int &kb) {
+    const int c = (int)blockIdx.x;
+    col = c % P.ncol;
+    const int part = c / P.ncol;
+    const int np = P.nplanes + P.split_bias;
+    const int b0 = max(0, min((part * np) / P.parts, P.nplanes));
+    const int b1 = part + 1 == P.parts ? P.nplanes : max(0, min(((part + 1) * np) / P.parts, P.nplanes));
+    ka = P.ka0 + b0;
+    kb = P.ka0 + b1;
+}
+
+// Producer warpgroup.  Warp TY: one lane issues the TMA loads -- planes 0..
+// STAGES-1 up front, then plane s+STAGES as soon as the consumers release
+// plane s (`empty`); it never waits for anything else, so a refill is never
+// held up behind aux work.  Warps TY+1..TY+3 (96 threads): for every plane,
+// once its tile has landed (`full`), rho_i / square of the tile + halo 1 into
+// the aux ring, then `afull` (count WS_AW).
+constexpr int WS_AW = WS_PW - 1;  // aux warps
+__device__ __forceinline__ void ws_producer(const CUtensorMap *umap, const CUtensorMap *fmap,
+                                            const Params &P) {
+    int col, ka, kb;
+    ws_segment(P, col, ka, kb);
+    if (ka >= kb) return;
+    const int i0 = 1 + (col % P.ntx) * TX, j0 = 1 + (col / P.ntx) * TY;
+    const int nu = kb - ka + 2;  // u planes ka .. kb+1
+    const int nf = kb - ka;      // forcing planes ka .. kb-1
+    const int warp = (int)threadIdx.x / 32, lane = (int)threadIdx.x % 32;
+    uint64_t *full = ws_full(), *afull = ws_afull();
+    if (warp == TY) {
+        if (lane != 0) return;
+        // in deadline order: step t reads u(t+2) (own column) and f(t)
+        for (int s = 0; s < WS_US && s < nu; ++s) ws_issue_u(umap, P, i0, j0, ka + s, s);
+        for (int s = 0; s < WS_FS && s < nf; ++s) ws_issue_f(fmap, P, i0, j0, ka + s, s);
+        for (int t = 0;; ++t) {
+            const int su_ = t + 2 + (WS_US - 2), sf = t + WS_FS;  // next u / f to issue
+            const bool mu = su_ < nu, mf = sf < nf;
+            if (!mu && !mf) break;
+            if (mu) {  // u(su_) reuses the slot of u(su_ - WS_US), released at step su_ - WS_US
+                const int r = su_ - WS_US;
+                ws_pwait(&ws_empty()[r % WS_US], (uint32_t)(r / WS_US) & 1u);
+                ws_issue_u(umap, P, i0, j0, ka + su_, su_ % WS_US);
+            }
+            if (mf) {
+                const int r = sf - WS_FS;
+                ws_pwait(&ws_fempty()[r % WS_FS], (uint32_t)(r / WS_FS) & 1u);
+                ws_issue_f(fmap, P, i0, j0, ka + sf, sf % WS_FS);
+            }
+        }
+        return;
+    }
+    const int pt = (int)threadIdx.x - (TY + 1) * 32;  // 0 .. 32*WS_AW-1
+    double2 *ax = ws_aux();
+    for (int s = 0; s < nu; ++s) {
+        const int slot = s % WS_US;
+        ws_pwait(&full[slot], (uint32_t)(s / WS_US) & 1u);
+        // rho_i, square of every point of the tile + halo 1 (App. A step 0)
+        const double *ut = ws_u() + (size_t)slot * U_SLOT;
+        double2 *at = ax + (size_t)slot * A_SLOT;
+        for (int p = pt; p < A_SLOT; p += WS_AW * 32) {
+            const int r = p / AXW, c = p - r * AXW;
+            const int ui = (r + 1) * UX + (c + HX - 1);
+            double rho, sq;
+            aux_of(ut[ui], ut[ui + UPM], ut[ui + 2 * UPM], ut[ui + 3 * UPM], rho, sq);
+            at[p] = make_double2(rho, sq);
+        }
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&afull[slot]);  // release: the aux stores above
+    }
+}
+
+// Consumer per-thread state (as rhs_kernel.cuh Seg, aux from smem).
+struct SegW {
+    double *rptr;
+    int uc, ac, fo;
+    bool active, mid_x;
+    int ycase;
+    int xo;
+    double a[3][5];
+    double rq, sq;   // rho_i / square of plane k-1 (planes k, k+1: from the aux ring)
+    double tp[5];
+};
+
+template <int R, bool UD>
+__device__ __forceinline__ void ws_step(SegW &g, const Params &P, int k, int q, int ka) {
+    constexpr int Q = R % 3, Z = (R + 1) % 3, PI = (R + 2) % 3;  // planes k-1, k, k+1
+    const Coef &C = P.c;
+    double *const su = ws_u();
+    const double2 *const ax = ws_aux();
+    const double *s = su + (size_t)(q % WS_US) * U_SLOT;
+    const double2 *a0 = ax + (size_t)(q % WS_US) * A_SLOT;
+    double acc[5];
+    {   // forcing(k): its own ring, released right after this read
+        mbar_wait(&ws_ffull()[q % WS_FS], (uint32_t)(q / WS_FS) & 1u);
+        const double *fs = ws_f() + (size_t)(q % WS_FS) * F_SLOT;
+#pragma unroll
+        for (int m = 0; m < 5; ++m) acc[m] = fs[m * TY * FX + g.fo];
+        __syncwarp();
+        if ((threadIdx.x & 31) == 0) mbar_arrive(&ws_fempty()[q % WS_FS]);
+    }
+    // the aux of plane k+1 (own rho_i / square for the zeta flux) is in place
+    // and plane k+2's tile has landed (own column read at the end of the
+    // step); plane k+2's aux is not needed yet, so its evaluation overlaps
+    // this step
+    mbar_wait(&ws_afull()[(q + 1) % WS_US], (uint32_t)((q + 1) / WS_US) & 1u);
+    mbar_wait(&ws_full()[(q + 2) % WS_US], (uint32_t)((q + 2) / WS_US) & 1u);
+    const double *const s2 = su + (size_t)((q + 2) % WS_US) * U_SLOT;
+    double an[5];
+    const double (&wz)[5] = g.a[Z];
+    const double2 own = a0[g.ac];  // rho_i / square of plane k
+    const double r0 = own.x, s0 = own.y;
+    double vc[3];
+    vc[0] = wz[1] * r0;
+    vc[1] = wz[2] * r0;
+    vc[2] = wz[3] * r0;
+    const double qsc = s0 * r0;
+    const double pc = wz[4] * r0;
+    auto zeta = [&]() {
+        Nb p, qn;
+#pragma unroll
+        for (int m = 0; m < 5; ++m) {
+            p.u[m] = g.a[PI][m];
+            qn.u[m] = g.a[Q][m];
+        }
+        const double2 o1 = ax[(size_t)((q + 1) % WS_US) * A_SLOT + g.ac];  // plane k+1
+        p.rho = o1.x; p.sq = o1.y;
+        qn.rho = g.rq; qn.sq = g.sq;
+        flux_dir<3, false, UD>(acc, wz, vc, qsc, pc, p, qn, C, 2);
+    };
+#if SAFARA_ZETA_FIRST
+    zeta();
+#endif
+    {   // xi: neighbours' rho_i / square from the aux tile
+        Nb p, qn;
+        load5(p.u, s, g.uc + 1);
+        load5(qn.u, s, g.uc - 1);
+        const double2 ap = a0[g.ac + 1], aq = a0[g.ac - 1];
+        p.rho = ap.x; p.sq = ap.y;
+        qn.rho = aq.x; qn.sq = aq.y;
+        double t[5];
+        {
+            double pp[5], qq[5];
+            if (g.mid_x) {
+                load5(pp, s, g.uc + 2);
+                load5(qq, s, g.uc - 2);
+                diss_terms<false>(t, qq, qn.u, wz, p.u, pp, Cases{});
+            } else {
+                const int xo = g.xo;
+                load5(pp, s, g.uc + (xo & 0xff));
+                load5(qq, s, g.uc - ((xo >> 8) & 0xff));
+                diss_terms_table(t, qq, qn.u, wz, p.u, pp, (xo & (1 << 16)) ? -4.0 : 0.0,
+                                 (xo & (1 << 17)) ? 5.0 : 6.0, (xo & (1 << 18)) ? -4.0 : 0.0);
+            }
+        }
+        flux_dir<1, false, UD>(acc, wz, vc, qsc, pc, p, qn, C, 0);
+        diss_apply(acc, t, C.dssp);
+    }
+    {   // eta
+        Nb p, qn;
+        load5(p.u, s, g.uc + UX);
+        load5(qn.u, s, g.uc - UX);
+        const double2 ap = a0[g.ac + AXW], aq = a0[g.ac - AXW];
+        p.rho = ap.x; p.sq = ap.y;
+        qn.rho = aq.x; qn.sq = aq.y;
+        double t[5];
+        {
+            double pp[5], qq[5];
+            load5(pp, s, g.uc + 2 * UX);
+            load5(qq, s, g.uc - 2 * UX);
+            diss_terms_case(t, qq, qn.u, wz, p.u, pp, g.ycase);
+        }
+        // every read of plane k's slot (u, forcing, aux) is done: release it
+        __syncwarp();
+        if ((threadIdx.x & 31) == 0) mbar_arrive(&ws_empty()[q % WS_US]);
+        flux_dir<2, false, UD>(acc, wz, vc, qsc, pc, p, qn, C, 1);
+        diss_apply(acc, t, C.dssp);
+    }
+#if !SAFARA_ZETA_FIRST
+    zeta();
+#endif
+    load5(an, s2, g.uc);
+    {
+        double t_z[5];
+        if (is_mid(k, P.nz)) {
+#pragma unroll
+            for (int m = 0; m < 5; ++m) t_z[m] = __fma_rn(-4.0, g.a[PI][m], g.tp[m]) + an[m];
+        } else {
+            const Cases c = cases_of(k, P.nz);
+#pragma unroll
+            for (int m = 0; m < 5; ++m) {
+                const double y1 = c.hp1 ? g.a[PI][m] : 0.0;
+                const double y2 = c.hp2 ? an[m] : 0.0;
+                t_z[m] = __fma_rn(-4.0, y1, g.tp[m]) + y2;
+            }
+        }
+        diss_apply(acc, t_z, C.dssp);
+    }
+    if (g.active) {
+        double *rp = g.rptr;
+#pragma unroll
+        for (int m = 0; m < 5; ++m) {
+            __stcs(rp, acc[m] * C.dt);
+            rp += SM(r);
+        }
+    }
+    g.rptr += SK(r);
+    zeta_partial(g.tp, g.a[Q], g.a[Z], g.a[PI], k + 1, P.nz, is_mid(k + 1, P.nz));
+#pragma unroll
+    for (int m = 0; m < 5; ++m) g.a[Q][m] = an[m];
+    g.rq = r0;  // plane k is plane k-1 of the next step
+    g.sq = s0;
+    (void)ka;
+}
+
+template <bool UD>
+__device__ __forceinline__ void ws_consumer(const Params &P) {
+    int col, ka, kb;
+    ws_segment(P, col, ka, kb);
+    if (ka >= kb) return;
+    const int tid = (int)threadIdx.x;
+    const int tx = tid % TX, ty = tid / TX;
+    const int i0 = 1 + (col % P.ntx) * TX, j0 = 1 + (col / P.ntx) * TY;
+    const int i = i0 + tx, j = j0 + ty;
+    const int nx_s = reread(P.nx), ny_s = reread(P.ny);
+    SegW g;
+    g.active = (i <= nx_s - 2) && (j <= ny_s - 2);
+    g.fo = ty * FX + tx + 1;
+    g.uc = (ty + 2) * UX + (tx + HX);
+    g.ac = (ty + 1) * AXW + (tx + 1);
+    g.mid_x = is_mid(i0, P.nx) && is_mid(i0 + TX - 1, P.nx);
+    {
+        const Cases cs = cases_of(i0 + tx, P.nx);
+        g.xo = (i0 + tx == P.nx - 3 ? 3 : 2) | ((i0 + tx == 2 ? 3 : 2) << 8) |
+               (cs.hm1 ? 1 << 16 : 0) | (cs.five ? 1 << 17 : 0) | (cs.hp1 ? 1 << 18 : 0);
+    }
+    g.ycase = is_mid(j, ny_s) ? 0 : j == 1 ? 1 : j == 2 ? 2 : j == ny_s - 3 ? 3 : 4;
+    g.rptr = P.r + ((idx_t)i + SY(r) * j + SK(r) * (ka - P.k0));
+    double *su = ws_u();
+    {   // window: planes ka-2, ka-1 from global memory, ka and ka+1 from the ring
+        const int ic = min(i, nx_s - 1), jc = min(j, ny_s - 1);
+        const int lk = ka - P.k0 + P.ukoff;
+        const double *uc0 = P.u + (idx_t)(ic + SY(u) * jc);
+#pragma unroll
+        for (int m = 0; m < 5; ++m)
+            g.a[0][m] = lk - 1 >= 0 ? __ldg(uc0 + SM(u) * m + SK(u) * (lk - 1)) : 0.0;
+        double am2[5];
+#pragma unroll
+        for (int m = 0; m < 5; ++m)
+            am2[m] = lk - 2 >= 0 ? __ldg(uc0 + SM(u) * m + SK(u) * (lk - 2)) : 0.0;
+        aux_of(g.a[0][0], g.a[0][1], g.a[0][2], g.a[0][3], g.rq, g.sq);
+        mbar_wait(&ws_afull()[0], 0u);
+        load5(g.a[1], su, g.uc);
+        zeta_partial(g.tp, am2, g.a[0], g.a[1], ka, P.nz, is_mid(ka, P.nz));
+        mbar_wait(&ws_full()[1], 0u);
+        load5(g.a[2], su + (size_t)1 * U_SLOT, g.uc);
+    }
+    int k = ka, q = 0;
+#pragma unroll 1
+    for (; k + 3 <= kb; k += 3, q += 3) {
+        ws_step<0, UD>(g, P, k, q, ka);
+        ws_step<1, UD>(g, P, k + 1, q + 1, ka);
+        ws_step<2, UD>(g, P, k + 2, q + 2, ka);
+    }
+    if (k < kb) {
+        ws_step<0, UD>(g, P, k, q, ka);
+        if (k + 1 < kb) ws_step<1, UD>(g, P, k + 1, q + 1, ka);
+    }
+}
+
+template <bool UD>
+__device__ __forceinline__ void rhs_body_ws(const CUtensorMap *umap, const CUtensorMap *fmap,
+                                            const Params &P) {
+    if ((int)blockIdx.x >= P.ncta) {  // the boundary faces (extra CTAs on idle SMs)
+        copy_faces<false>(P, (int)blockIdx.x - P.ncta, P.nface_cta);
+        return;
+    }
+    const int tid = (int)threadIdx.x;
+    if (tid == 0) {
+        prefetch_tmap(umap);
+        prefetch_tmap(fmap);
+        for (int s = 0; s < WS_US; ++s) {
+            mbar_init(&ws_full()[s], 1);
+            mbar_init(&ws_afull()[s], WS_AW);
+            mbar_init(&ws_empty()[s], TY);
+        }
+        for (int s = 0; s < WS_FS; ++s) {
+            mbar_init(&ws_ffull()[s], 1);
+            mbar_init(&ws_fempty()[s], TY);
+        }
+        fence_mbar_init();
+    }
+    __syncthreads();
+    if (P.nface_cta == 0) copy_faces<false>(P, (int)blockIdx.x, P.ncta);
+    if (tid >= TY * 32) {
+        setmaxnreg_dec_producer();
+        ws_producer(umap, fmap, P);
+    } else {
+        setmaxnreg_inc_consumer();
+        ws_consumer<UD>(P);
+    }
+}
+
+}  // namespace dev
+}  // namespace safara

@@ -131,6 +131,15 @@ int err_norm_grid();
 cudaError_t launch_error_norm(const double *u, const double *ue, int nx, int ny, int nz, int sy,
                               int sm, int sk, double *work, double *rms, cudaStream_t s);
 
+// Round 2: the warp-specialised kernels (rhs_ws.cuh; one segment per CTA, no
+// aux output, no peer halo).  attr: 2 entries (uniform d1, general).
+cudaError_t launch_rhs_ws_fast(const CUtensorMap &umap, const CUtensorMap &fmap, const Params &p,
+                               bool uniform_d, cudaStream_t s);
+cudaError_t launch_rhs_ws_strict(const CUtensorMap &umap, const CUtensorMap &fmap, const Params &p,
+                                 bool uniform_d, cudaStream_t s);
+cudaError_t setup_rhs_ws_fast(cudaFuncAttributes *attr);
+cudaError_t setup_rhs_ws_strict(cudaFuncAttributes *attr);
+
 // attr: 4 entries (production NAS path, general coefficients, aux, NAS + aux)
 cudaError_t setup_rhs_fast(int *ctas_per_sm, cudaFuncAttributes *attr);
 cudaError_t setup_rhs_strict(int *ctas_per_sm, cudaFuncAttributes *attr);

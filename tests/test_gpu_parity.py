@@ -256,3 +256,42 @@ def test_analytic_navier_stokes_field(shape):
     o = oracle.compute_rhs(u, f, dt=1e-3, threads=8)
     assert np.array_equal(gpu_rhs(u, f, 1e-3, strict=True), o)
     assert_tol(gpu_rhs(u, f, 1e-3, strict=False), o)
+
+
+_WS_SCRIPT = r"""
+import sys, numpy as np, torch
+sys.path.insert(0, {root!r})
+import nasgen, oracle, paper_conf_icpp_tiankexc16_b200 as sr
+sr.init(0)
+for bench, cls in (("BT", "S"), ("SP", "W"), ("BT", "A"), ("BT", "C")):
+    inp = nasgen.make_class(bench, cls, seed=1, B=1e-2)
+    nz, ny, nx, _ = inp.u.shape
+    c = sr.coeffs_nas(nx, ny, nz, inp.dt)
+    du, df = sr.pack(inp.u), sr.pack(inp.forcing)
+    o = oracle.compute_rhs(inp.u, inp.forcing, dt=inp.dt, threads=8)
+    for strict in (True, False):
+        dr = torch.full_like(du, float("nan"))
+        sr.rhs(du, df, dr, nx, c, strict=strict)
+        torch.cuda.synchronize()
+        g = sr.unpack(dr, nx)
+        if strict:
+            assert np.array_equal(g, o), (bench, cls)
+        else:
+            assert (np.abs(g - o) <= 1e-12 * np.abs(o) + 1e-14).all(), (bench, cls)
+print("ws ok")
+"""
+
+
+def test_warp_specialised_kernel_parity():
+    """The warp-specialised kernel (rhs_ws.cuh, SAFARA_WS=1: producer
+    warpgroup computing rho_i/square into a shared-memory aux ring) is held to
+    the same bar: STRICT bit-identical, production within c5 (own process:
+    the knob is read once at init)."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, "-c", _WS_SCRIPT.format(root=root)],
+                       env=dict(os.environ, SAFARA_WS="1"), capture_output=True, text=True,
+                       timeout=600)
+    assert r.returncode == 0 and "ws ok" in r.stdout, r.stderr[-2000:]
