@@ -60,7 +60,7 @@ struct Tune {
     int split_bias = 0;  // experiments: shift the lockstep k-split points (no peer)
     int peer_bias_maxpart = 6;  // peer_bias only for k-parts of at most this many planes
     int peer_timeout_ms = 30000;  // f2 flag waits: give up and trap after this long
-    int ws = 0;  // 1: warp-specialised kernel (rhs_ws.cuh) where it applies (A/B: 1-2 % slower, off)
+    int ws = 1;  // warp-specialised kernel (rhs_ws.cuh) where it applies (0: round-1 kernel)
 } g_tune;
 
 int env_int(const char *name, int dflt) {
@@ -789,6 +789,20 @@ int safara_kernel_info(int which, safara_kernel_info_t *out) {
     int rc = current_device(&dev);
     if (rc) return rc;
     const DeviceState &st = g_dev[dev];
+    if (g_tune.ws) {
+        // the warp-specialised kernel (one-segment lockstep launches, e.g.
+        // every full-grid pass at class C): NAS coefficients instantiation
+        const cudaFuncAttributes *a = which ? st.attr_ws_strict : st.attr_ws_fast;
+        out->regs_per_thread = a[0].numRegs;  // launch allocation (setmaxnreg moves them)
+        out->local_bytes = (int)a[0].localSizeBytes;
+        out->smem_bytes = (int)(a[0].sharedSizeBytes + WS_SMEM_BYTES);
+        out->threads_per_cta = WS_THREADS;
+        out->ctas_per_sm = 1;
+        out->tile_x = TX;
+        out->tile_y = TY;
+        out->stages = WS_US;
+        return SAFARA_OK;
+    }
     const cudaFuncAttributes *a = which ? st.attr_strict : st.attr_fast;
     out->regs_per_thread = a[0].numRegs;
     // local (spill) bytes of the production instantiation (NAS coefficients,

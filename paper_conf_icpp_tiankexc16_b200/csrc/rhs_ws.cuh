@@ -32,10 +32,6 @@
 namespace safara {
 namespace dev {
 
-constexpr int WS_PW = 4;                     // producer warps (one warpgroup)
-constexpr int WS_THREADS = (TY + WS_PW) * 32;
-constexpr int AXW = TX + 2, AYW = TY + 2;    // aux tile: columns i0-1..i0+TX, rows j0-1..j0+TY
-constexpr int A_SLOT = AXW * AYW;            // double2 per aux slot
 #ifndef SAFARA_WS_SLEEP
 #define SAFARA_WS_SLEEP 20000   // producer waits: suspend-time hint (ns), 0 = plain try_wait
 #endif
@@ -46,36 +42,6 @@ __device__ __forceinline__ void ws_pwait(uint64_t *bar, uint32_t parity) {
     mbar_wait(bar, parity);
 #endif
 }
-#ifndef SAFARA_WS_PREG
-#define SAFARA_WS_PREG 32                    // producer registers after setmaxnreg.dec
-#endif
-// consumer registers after setmaxnreg.inc: the rest of the 64K register file
-constexpr int WS_CREG = ((65536 / 32 - WS_PW * SAFARA_WS_PREG) / TY) / 8 * 8;
-static_assert(WS_CREG >= 128 && WS_CREG <= 256, "consumer register budget");
-
-// Shared memory: a u ring of WS_US plane tiles (with halo 2), the aux ring
-// (one (rho_i, square) tile per u slot) and a separate, shallower forcing ring
-// of WS_FS slots -- forcing(k) is read only at step k, u(k) already at step
-// k-2 (own column), so splitting the rings buys one more u plane of TMA
-// lookahead in the same shared memory.
-#ifndef SAFARA_WS_US
-#define SAFARA_WS_US 5
-#endif
-#ifndef SAFARA_WS_FS
-#define SAFARA_WS_FS 3
-#endif
-constexpr int WS_US = SAFARA_WS_US, WS_FS = SAFARA_WS_FS;
-constexpr size_t WS_U_BYTES = (size_t)WS_US * U_SLOT * 8;
-// (padded: the forcing ring behind it is a TMA destination, 128-byte aligned)
-constexpr size_t WS_AUX_BYTES = ((size_t)WS_US * A_SLOT * 16 + 127) / 128 * 128;
-constexpr size_t WS_F_BYTES = (size_t)WS_FS * F_SLOT * 8;
-constexpr size_t WS_BAR_OFF = WS_U_BYTES + WS_AUX_BYTES + WS_F_BYTES;
-constexpr size_t WS_SMEM_BYTES = WS_BAR_OFF + (3 * WS_US + 2 * WS_FS) * 8;
-static_assert(WS_SMEM_BYTES <= 227 * 1024, "WS shared memory");
-static_assert(WS_U_BYTES % 128 == 0 && (U_SLOT * 8) % 128 == 0 && (F_SLOT * 8) % 128 == 0 &&
-                  (WS_U_BYTES + WS_AUX_BYTES) % 128 == 0,
-              "TMA destinations 128-byte aligned");
-
 __device__ __forceinline__ double *ws_u() { return reinterpret_cast<double *>(smem_raw); }
 __device__ __forceinline__ double2 *ws_aux() {
     return reinterpret_cast<double2 *>(smem_raw + WS_U_BYTES);

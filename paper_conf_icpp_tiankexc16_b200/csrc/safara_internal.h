@@ -42,6 +42,43 @@ static_assert(STAGES * (8 + 4) <= XCOEF_OFF * 8, "mbarriers + release counters f
 constexpr size_t SMEM_BYTES = (size_t)STAGES * SLOT * 8 + (XCOEF_OFF + 3 * TX + TX / 2) * 8;
 constexpr int MIN_PLANES_PER_CTA = 2;  // small slabs: more k-parts win (SP-B/8: 16.4 -> 12.5 us, profiles/slab_sim_r01.txt)
 
+// Round 2 warp-specialised kernel (rhs_ws.cuh): TY consumer warps + one
+// producer warpgroup; u / aux / forcing rings in shared memory.
+constexpr int WS_PW = 4;                     // producer warps (one warpgroup)
+constexpr int WS_THREADS = (TY + WS_PW) * 32;
+constexpr int AXW = TX + 2, AYW = TY + 2;    // aux tile: columns i0-1..i0+TX, rows j0-1..j0+TY
+constexpr int A_SLOT = AXW * AYW;            // double2 per aux slot
+#ifndef SAFARA_WS_PREG
+#define SAFARA_WS_PREG 32                    // producer registers after setmaxnreg.dec
+#endif
+// consumer registers after setmaxnreg.inc: the rest of the 64K register file
+constexpr int WS_CREG = ((65536 / 32 - WS_PW * SAFARA_WS_PREG) / TY) / 8 * 8;
+static_assert(WS_CREG >= 128 && WS_CREG <= 256, "consumer register budget");
+
+// Shared memory: a u ring of WS_US plane tiles (with halo 2), the aux ring
+// (one (rho_i, square) tile per u slot) and a separate, shallower forcing ring
+// of WS_FS slots -- forcing(k) is read only at step k, u(k) already at step
+// k-2 (own column), so splitting the rings buys one more u plane of TMA
+// lookahead in the same shared memory.
+#ifndef SAFARA_WS_US
+#define SAFARA_WS_US 4
+#endif
+#ifndef SAFARA_WS_FS
+#define SAFARA_WS_FS 2
+#endif
+constexpr int WS_US = SAFARA_WS_US, WS_FS = SAFARA_WS_FS;
+constexpr size_t WS_U_BYTES = (size_t)WS_US * U_SLOT * 8;
+// (padded: the forcing ring behind it is a TMA destination, 128-byte aligned)
+constexpr size_t WS_AUX_BYTES = ((size_t)WS_US * A_SLOT * 16 + 127) / 128 * 128;
+constexpr size_t WS_F_BYTES = (size_t)WS_FS * F_SLOT * 8;
+constexpr size_t WS_BAR_OFF = WS_U_BYTES + WS_AUX_BYTES + WS_F_BYTES;
+constexpr size_t WS_SMEM_BYTES = WS_BAR_OFF + (3 * WS_US + 2 * WS_FS) * 8;
+static_assert(WS_SMEM_BYTES <= 227 * 1024, "WS shared memory");
+static_assert(WS_U_BYTES % 128 == 0 && (U_SLOT * 8) % 128 == 0 && (F_SLOT * 8) % 128 == 0 &&
+                  (WS_U_BYTES + WS_AUX_BYTES) % 128 == 0,
+              "TMA destinations 128-byte aligned");
+
+
 // Device-side coefficients: safara_coeffs_t plus the constant products that
 // the NAS text evaluates left to right (xxcon2*con43 -> one double).
 struct Coef {
