@@ -50,6 +50,8 @@ def parse():
                          "PAPER.md Fig. 8 loop (f4) on --seismic-n^3")
     ap.add_argument("--seismic-n", type=int, default=256)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-other-configs", action="store_true",
+                    help="skip the rotating-buffer SP-B / BT-A / SP-W lines")
     ap.add_argument("--halo", default="peer", choices=["peer", "nccl"],
                     help="N>1: peer = halo fused into the kernel (loads from the neighbours' "
                          "slabs over NVLink, SURVEY f2); nccl = NCCL send/recv exchange "
@@ -80,6 +82,28 @@ def measured_peaks():
             d = json.load(fh)
         return float(d["hbm_gbs"]), "measured"
     return 6650.0, "fallback"
+
+
+def fp64_peak():
+    """Measured DFMA peak (TFLOP/s) from the committed microbenchmark
+    (tools/micro/fp64_peak.cu -> profiles/fp64_micro_r01.txt), else the
+    nominal 148 SMs x 64 FP64 FMA/clk x 2 x 1.965 GHz."""
+    import re
+    p = os.path.join(ROOT, "profiles", "fp64_micro_r01.txt")
+    if os.path.exists(p):
+        vals = [float(m) for m in re.findall(r"DFMA throughput: .*?: ([0-9.]+) TFLOP/s",
+                                             open(p).read())]
+        if vals:
+            return max(vals), "measured (profiles/fp64_micro_r01.txt, DFMA microbenchmark)"
+    return 148 * 64 * 2 * 1.965e9 / 1e12, "nominal"
+
+
+def ncu_entry(config_key):
+    p = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    if not os.path.exists(p):
+        return {}
+    with open(p) as fh:
+        return json.load(fh).get(config_key, {})
 
 
 def ncu_traffic(config_key):
@@ -158,7 +182,7 @@ class ClockSampler:
                 "reasons": sorted(reasons)}
 
 
-def cpu_oracle_time(inp, max_seconds=12.0, threads=None):
+def cpu_oracle_time(inp, max_seconds=12.0, threads=None, min_passes=1):
     """Time the oracle as it stands on the host cores (full passes)."""
     import oracle
     threads = threads or os.cpu_count() or 1
@@ -168,12 +192,68 @@ def cpu_oracle_time(inp, max_seconds=12.0, threads=None):
         oracle.compute_rhs(inp.u, inp.forcing, dt=inp.dt, threads=threads)
         n += 1
         el = time.perf_counter() - t0
-        if el >= max_seconds or n >= 50:
+        if (el >= max_seconds and n >= min_passes) or n >= 50:
             break
     pts = inp.nx * inp.ny * inp.nz
     return {"value": pts * n / el / 1e9, "unit": "Gpt/s", "cores": threads, "kind": "oracle",
             "sample": f"{n} full {inp.nx}x{inp.ny}x{inp.nz} passes (plain C, -O2, "
                       f"-ffp-contract=off, OpenMP over k) in {el:.2f} s"}
+
+
+def cpu_baseline(inp):
+    """The oracle on all host cores (the reported baseline) and on ONE core
+    (GPU vs one core), each a bounded sample of full passes."""
+    full = cpu_oracle_time(inp, max_seconds=9.0)
+    one = cpu_oracle_time(inp, max_seconds=6.0, threads=1)
+    full["single_thread"] = {k: one[k] for k in ("value", "unit", "cores", "sample")}
+    try:
+        model = [l.split(":", 1)[1].strip() for l in open("/proc/cpuinfo")
+                 if l.startswith("model name")][0]
+    except (OSError, IndexError):
+        model = "unknown"
+    full["cpu"] = model
+    return full
+
+
+def other_configs(args, sr, torch, stream):
+    """BASELINE.json's other configs, timed the same way but with ROTATING
+    input sets whose total exceeds 2x the 126 MB L2, so each
+    pass reads its inputs from HBM: these small grids are L2/launch-bound
+    and reported as such (not the headline)."""
+    import nasgen
+    out = []
+    l2 = 126e6
+    for bench, cls in (("SP", "B"), ("BT", "A"), ("SP", "W")):
+        n, dt = nasgen.CLASSES[(bench, cls)]
+        inp = nasgen.make_class(bench, cls, seed=1)
+        c = sr.coeffs_nas(n, n, n, dt)
+        du, df = sr.pack(inp.u), sr.pack(inp.forcing)
+        set_bytes = 3 * du.numel() * 8
+        nsets = max(2, int(2 * l2 // set_bytes) + 1)
+        sets = [(du.clone(), df.clone(), torch.empty_like(du)) for _ in range(nsets)]
+        del du, df
+        for k in range(3 * nsets):
+            u, f, r = sets[k % nsets]
+            sr.rhs(u, f, r, n, c, stream=stream)
+        steps = max(args.steps, 10 * nsets)
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for k in range(steps):
+            u, f, r = sets[k % nsets]
+            sr.rhs(u, f, r, n, c, stream=stream)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        ms = e0.elapsed_time(e1) / steps
+        pts = n ** 3
+        out.append({"workload": nasgen.config_name(bench, cls), "value": pts / (ms * 1e-3) / 1e9,
+                    "unit": "Gpt/s", "us_per_pass": ms * 1e3,
+                    "hbm_frac": BYTES_PER_POINT * pts / (ms * 1e-3) / 1e9 / measured_peaks()[0],
+                    "l2": f"rotating {nsets} input sets of {set_bytes / 1e6:.1f} MB "
+                          f"({nsets * set_bytes / 1e6:.0f} MB > 2x L2)",
+                    "bound": "L2/launch-bound (small grid), effective throughput"})
+        del sets
+    return out
 
 
 def config_of(args):
@@ -218,7 +298,10 @@ def run_reference(args):
         "config": {"workload": nasgen.config_name(bench, cls), "grid": [n, n, n],
                    "points": pts, "l2": "host"},
         "cpu_baseline": {"value": value, "unit": "Gpt/s", "cores": threads, "kind": "oracle",
-                         "sample": f"{args.steps} full {n}^3 passes of the plain-C oracle"},
+                         "sample": f"{args.steps} full {n}^3 passes of the plain-C oracle",
+                         "single_thread": {k: v for k, v in cpu_oracle_time(
+                             inp, max_seconds=6.0, threads=1).items()
+                             if k in ("value", "unit", "cores", "sample")}},
         "e2e": {"value": value, "unit": "Gpt/s", "h2d_bytes_per_step": 0,
                 "d2h_bytes_per_step": 0},
     }
@@ -314,6 +397,9 @@ def run_single(args):
     peak, peak_kind = measured_peaks()
     key = f"{bench}-{cls}"
     traffic = ncu_traffic(key)
+    fpk, fpk_kind = fp64_peak()
+    ncu_e = ncu_entry(key)
+    fp64_tf = FLOPS_PER_POINT * pts / (kern_ms * 1e-3) / 1e12
 
     # e2e: host (pinned) buffers through the C ABI, H2D + pass + D2H per step
     e2e_ms, nbytes = float("nan"), 0
@@ -350,6 +436,12 @@ def run_single(args):
                      "frac": achieved / peak, "peak_kind": peak_kind, "traffic": traffic,
                      "bytes_per_point": bytes_per_point, "kernel_ms": kern_ms,
                      "frac_of_8000": achieved / 8000.0},
+        "roofline_fp64": {"bound": "fp64", "achieved": fp64_tf, "peak": fpk,
+                          "unit": "TFLOP/s", "frac": fp64_tf / fpk, "peak_kind": fpk_kind,
+                          "flops_per_point": FLOPS_PER_POINT,
+                          "ncu_fp64_pipe_active_pct": ncu_e.get("fp64_pipe_active_pct"),
+                          "note": "algorithmic flops (430/pt); the FP64 pipe is the "
+                                  "near-binding second roofline (DESIGN.md §5)"},
         "clocks": clocks,
         "e2e": {"value": pts / (e2e_ms * 1e-3) / 1e9, "unit": "Gpt/s",
                 "h2d_bytes_per_step": 2 * nbytes, "d2h_bytes_per_step": nbytes,
@@ -357,8 +449,10 @@ def run_single(args):
         "gpu_launches": launches,
         "kernel": sr.kernel_info(args.strict),
     }
+    if not args.no_other_configs and args.workload == "rhs" and not args.grid:
+        line["other_configs"] = other_configs(args, sr, torch, stream)
     if not args.no_cpu_baseline:
-        line["cpu_baseline"] = cpu_oracle_time(inp)
+        line["cpu_baseline"] = cpu_baseline(inp)
     print(json.dumps(line), flush=True)
 
 

@@ -126,15 +126,17 @@ __device__ __forceinline__ void ws_producer(const CUtensorMap *umap, const CUten
             const int su_ = t + 2 + (WS_US - 2), sf = t + WS_FS;  // next u / f to issue
             const bool mu = su_ < nu, mf = sf < nf;
             if (!mu && !mf) break;
+            // step t releases forcing(t) at its start and u(t) after its
+            // eta stencil: refill in that order
+            if (mf) {  // f(sf) reuses the slot of f(sf - WS_FS), released at step sf - WS_FS
+                const int r = sf - WS_FS;
+                ws_pwait(&ws_fempty()[r % WS_FS], (uint32_t)(r / WS_FS) & 1u);
+                ws_issue_f(fmap, P, i0, j0, ka + sf, sf % WS_FS);
+            }
             if (mu) {  // u(su_) reuses the slot of u(su_ - WS_US), released at step su_ - WS_US
                 const int r = su_ - WS_US;
                 ws_pwait(&ws_empty()[r % WS_US], (uint32_t)(r / WS_US) & 1u);
                 ws_issue_u(umap, P, i0, j0, ka + su_, su_ % WS_US);
-            }
-            if (mf) {
-                const int r = sf - WS_FS;
-                ws_pwait(&ws_fempty()[r % WS_FS], (uint32_t)(r / WS_FS) & 1u);
-                ws_issue_f(fmap, P, i0, j0, ka + sf, sf % WS_FS);
             }
         }
         return;
@@ -357,11 +359,42 @@ __device__ __forceinline__ void ws_consumer(const Params &P) {
     }
 }
 
+// SAFARA_TIMELINE builds: {start, end, smid | cycles << 16} of this CTA
+// (thread 0 at the end of its role; consumers' warp 0 for compute CTAs).
+__device__ __forceinline__ void ws_timeline(const Params &P, unsigned long long t_start,
+                                            long long c_start) {
+#ifdef SAFARA_TIMELINE
+    if (P.dbg) {
+        unsigned long long t_end;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_end));
+        unsigned smid;
+        asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+        P.dbg[3 * blockIdx.x] = t_start;
+        P.dbg[3 * blockIdx.x + 1] = t_end;
+        P.dbg[3 * blockIdx.x + 2] = smid | ((unsigned long long)(clock64() - c_start) << 16);
+    }
+#else
+    (void)P; (void)t_start; (void)c_start;
+#endif
+}
+
 template <bool UD>
 __device__ __forceinline__ void rhs_body_ws(const CUtensorMap *umap, const CUtensorMap *fmap,
                                             const Params &P) {
+    unsigned long long t_start = 0;
+    long long c_start = 0;
+#ifdef SAFARA_TIMELINE
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_start));
+    c_start = clock64();
+#endif
+    // PDL (SAFARA_PDL builds): the next pass on the stream may be scheduled
+    // now; every global access below waits for the previous grid.
+    grid_dep_launch();
     if ((int)blockIdx.x >= P.ncta) {  // the boundary faces (extra CTAs on idle SMs)
+        grid_dep_wait();
         copy_faces<false>(P, (int)blockIdx.x - P.ncta, P.nface_cta);
+        __syncthreads();
+        if (threadIdx.x == 0) ws_timeline(P, t_start, c_start);
         return;
     }
     const int tid = (int)threadIdx.x;
@@ -380,6 +413,7 @@ __device__ __forceinline__ void rhs_body_ws(const CUtensorMap *umap, const CUten
         fence_mbar_init();
     }
     __syncthreads();
+    grid_dep_wait();
     if (P.nface_cta == 0) copy_faces<false>(P, (int)blockIdx.x, P.ncta);
     if (tid >= TY * 32) {
         setmaxnreg_dec_producer();
@@ -387,6 +421,7 @@ __device__ __forceinline__ void rhs_body_ws(const CUtensorMap *umap, const CUten
     } else {
         setmaxnreg_inc_consumer();
         ws_consumer<UD>(P);
+        if (tid == 0) ws_timeline(P, t_start, c_start);
     }
 }
 

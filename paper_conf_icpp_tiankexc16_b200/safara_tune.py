@@ -212,7 +212,7 @@ def time_variant(tag_defines, steps: int = 100) -> float | None:
     b.build(force=True, extra=defines, out=out)
     env = dict(os.environ, SAFARA_LIB=out)
     res = subprocess.run([sys.executable, os.path.join(b.ROOT, "bench.py"), "--steps", str(steps),
-                          "--warmup", "10", "--no-cpu-baseline", "--soak-s", "0.3",
+                          "--warmup", "10", "--no-cpu-baseline", "--no-other-configs", "--soak-s", "0.3",
                           "--e2e-steps", "0"], capture_output=True, text=True, env=env)
     try:
         return json.loads(res.stdout.strip().splitlines()[-1])["roofline"]["kernel_ms"] * 1e3

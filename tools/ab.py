@@ -49,7 +49,7 @@ def run(reps, specs, steps=400):
                 k, _, v = e.partition("=")
                 env[k] = v
             r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--steps", str(steps),
-                                "--warmup", "20", "--no-cpu-baseline", "--e2e-steps", "1"],
+                                "--warmup", "20", "--no-cpu-baseline", "--no-other-configs", "--e2e-steps", "1"],
                                capture_output=True, text=True, env=env, timeout=600)
             try:
                 d = json.loads(r.stdout.strip().splitlines()[-1])
