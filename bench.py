@@ -44,7 +44,7 @@ def parse():
     ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--e2e-chunks", type=int, default=8,
                     help="k-chunks of the pipelined H2D / compute / D2H e2e path")
-    ap.add_argument("--workload", default="rhs", choices=["rhs", "rhs_aux", "seismic_dz"],
+    ap.add_argument("--workload", default="rhs", choices=["rhs", "rhs_aux", "rhs_norm", "rhs_aux_norm", "seismic_dz"],
                     help="rhs: the headline compute_rhs pass; rhs_aux: the same pass also "
                          "writing the 6 step-0 fields (SURVEY §8(f) f1); seismic_dz: the "
                          "PAPER.md Fig. 8 loop (f4) on --seismic-n^3")
@@ -334,6 +334,16 @@ def run_single(args):
 
         def step(st=None):
             sr.rhs_aux(du, df, dr, da, nx, c, strict=args.strict, stream=st or stream)
+    elif args.workload in ("rhs_norm", "rhs_aux_norm"):
+        # f1: rhs_norm accumulated in the store epilogue (+ the aux fields)
+        da = sr.empty_aux(nx, ny, nz, sr.SAFARA_AUX_BT) if args.workload == "rhs_aux_norm" else None
+        if da is not None:
+            bytes_per_point += 8 * sr.SAFARA_AUX_BT
+        rms_out = torch.empty(5, dtype=torch.float64, device="cuda")
+
+        def step(st=None):
+            sr.rhs_fused(du, df, dr, nx, c, aux=da, rms=rms_out, strict=args.strict,
+                         stream=st or stream)
     else:
         def step(st=None):
             sr.rhs(du, df, dr, nx, c, strict=args.strict, stream=st or stream)

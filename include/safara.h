@@ -321,6 +321,26 @@ int safara_rhs_slab_aux(const double *u_slab, const double *forcing_slab,
                         const safara_coeffs_t *coeffs, int flags, int part,
                         void *stream);
 
+/* One pass with the optional f1 outputs fused in: aux (NULL = none; naux as
+ * safara_rhs_aux) and the NPB rhs_norm of the result (rms NULL = none; else
+ * 5 device doubles rms[m] = sqrt(sum over interior points of rhs_m^2 /
+ * ((nx-2)(ny-2)(nz-2))), work: safara_norm_work_doubles() + 8 device
+ * doubles whose first word must be ZERO before the first call -- every call
+ * leaves it zero again).  The norm is accumulated in the store epilogue of
+ * the warp-specialised kernel (per-thread sums over its k march, warp trees,
+ * per-CTA partials) and finished by the last CTA to complete (an atomic
+ * counter in work[0]), which sums the CTA partials in CTA order -- one
+ * launch, no re-read of rhs; deterministic for a given grid.  Where that
+ * kernel does not apply (general coefficients, SAFARA_WS=0, non-lockstep
+ * decompositions) the library runs safara_rhs_rms after the pass instead
+ * (same contract, rhs re-read, 2 more launches).  Full grid, canonical-compatible
+ * descriptor; errors as safara_rhs_aux plus SAFARA_ERR_ARG (rms without
+ * work, overlaps).  Asynchronous.                                          */
+int safara_rhs_fused(const double *u, const double *forcing, double *rhs,
+                     double *aux, int naux, double *work, double *rms,
+                     const safara_dims_t *dims, const safara_coeffs_t *coeffs,
+                     int flags, void *stream);
+
 /* The NAS rhs_norm numerator (NPB error.f): out[m] = sum of rhs(m,i,j,k)^2
  * over the INTERIOR points (1 <= i <= nx-2, 1 <= j <= ny-2, 1 <= k <= nz-2)
  * of the planes this buffer holds: rhs has nzl planes, plane p = global

@@ -106,6 +106,8 @@ _SIGS = {
                          ctypes.c_int),
     "safara_seismic_dz": ([_dp] * 4 + [ctypes.POINTER(Dims3), ctypes.c_double, _dp], ctypes.c_int),
     "safara_rhs_rms": ([_dp, ctypes.POINTER(Dims), _dp, _dp, _dp], ctypes.c_int),
+    "safara_rhs_fused": ([_dp, _dp, _dp, _dp, ctypes.c_int, _dp, _dp, ctypes.POINTER(Dims),
+                          ctypes.POINTER(Coeffs), ctypes.c_int, _dp], ctypes.c_int),
     "safara_get_unique_id": ([ctypes.c_char_p], ctypes.c_int),
     "safara_shard_init": ([ctypes.c_char_p, ctypes.c_int, ctypes.c_int, ctypes.c_int,
                            ctypes.POINTER(ctypes.c_void_p)], ctypes.c_int),

@@ -183,7 +183,8 @@ int launch(const double *u, const double *f, double *r, const safara_dims_t &d, 
            int k0,
            int ukoff, int ka0, int kb0, int ka1, int kb1, int fk_lo, int fk_hi,
            const safara_coeffs_t *coeffs, int flags, cudaStream_t stream,
-           double *aux = nullptr, int naux = 0, int ska = 0, const PeerCfg *peer = nullptr) {
+           double *aux = nullptr, int naux = 0, int ska = 0, const PeerCfg *peer = nullptr,
+           double *norm_work = nullptr, double *norm_out = nullptr, bool *fused = nullptr) {
     int dev;
     int rc = current_device(&dev);
     if (rc) return rc;
@@ -344,7 +345,17 @@ int launch(const double *u, const double *f, double *r, const safara_dims_t &d, 
     // the warp-specialised kernel serves launches whose CTAs each own one
     // (column tile, k range) segment: lockstep over a single plane range,
     // without the f1 aux output or the f2 peer halo
-    const bool ws = g_tune.ws && lockstep && p.parts > 0 && p.n0 == p.nplanes && !aux && !peer;
+    const bool ws = g_tune.ws && lockstep && p.parts > 0 && p.n0 == p.nplanes && !peer;
+    // f1 fused rhs_norm: the warp-specialised kernel with NAS coefficients
+    // writes per-CTA partial sums; otherwise the caller runs the two-pass norm
+    if (fused) *fused = norm_work != nullptr && ws && ud;
+    if (fused && *fused) {
+        // work[0]: CTA counter (zero between passes), partials from work + 8
+        p.norm_ctr = reinterpret_cast<unsigned long long *>(norm_work);
+        p.norm_part = norm_work + 8;
+        p.norm_out = norm_out;
+        p.norm_npts = (double)(d.nx - 2) * (double)(d.ny - 2) * (double)(d.nz - 2);
+    }
     cudaError_t e;
     if (ws)
         e = strict ? launch_rhs_ws_strict(umap, fmap, p, ud, stream)
@@ -644,6 +655,43 @@ int safara_rhs_aux(const double *u, const double *forcing, double *rhs, double *
     const int nz = dims->nz;
     return launch(u, forcing, rhs, *dims, nz, nz, 0, 0, 1, nz - 1, 0, 0, 0, nz, coeffs, flags,
                   (cudaStream_t)stream, aux, naux, ska);
+}
+
+int safara_rhs_fused(const double *u, const double *forcing, double *rhs, double *aux, int naux,
+                     double *work, double *rms, const safara_dims_t *dims,
+                     const safara_coeffs_t *coeffs, int flags, void *stream) {
+    int rc = validate(dims, dims ? dims->nz : 0);
+    if (rc) return rc;
+    const long long bytes = (max_offset(*dims, dims->nz) + 1) * (long long)sizeof(double);
+    rc = check_ptrs(u, bytes, forcing, bytes, rhs, bytes);
+    if (rc) return rc;
+    int ska = 0;
+    if (aux) {
+        long long abytes;
+        rc = aux_layout(*dims, naux, dims->nz, &ska, &abytes);
+        if (rc) return rc;
+        rc = check_aux(aux, abytes, u, bytes, forcing, bytes, rhs, bytes);
+        if (rc) return rc;
+    } else {
+        naux = 0;
+    }
+    if (rms) {
+        if (!work) return SAFARA_ERR_ARG;
+        if (((uintptr_t)work | (uintptr_t)rms) & 7u) return SAFARA_ERR_ALIGN;
+        const long long wbytes = ((long long)safara_norm_work_doubles() + 8) * 8;
+        if (overlaps(work, wbytes, rhs, bytes) || overlaps(work, wbytes, u, bytes) ||
+            overlaps(work, wbytes, forcing, bytes) || overlaps(rms, 40, rhs, bytes) ||
+            overlaps(rms, 40, work, wbytes))
+            return SAFARA_ERR_ARG;
+    }
+    const int nz = dims->nz;
+    bool fused = false;
+    rc = launch(u, forcing, rhs, *dims, nz, nz, 0, 0, 1, nz - 1, 0, 0, 0, nz, coeffs, flags,
+                (cudaStream_t)stream, aux, naux, ska, nullptr, rms ? work : nullptr, rms,
+                rms ? &fused : nullptr);
+    if (rc || !rms || fused) return rc;
+    // not the warp-specialised NAS path: the two-pass norm (work[0] untouched)
+    return safara_rhs_rms(rhs, dims, work + 8, rms, stream);
 }
 
 int safara_rhs_slab_aux(const double *u_slab, const double *forcing_slab, double *rhs_slab,

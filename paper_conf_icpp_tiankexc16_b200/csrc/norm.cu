@@ -88,6 +88,12 @@ cudaError_t launch_sumsq(const double *rhs, int nx, int ny, int sy, int sm, int 
     return cudaGetLastError();
 }
 
+cudaError_t launch_partials_final(const double *work, int G, double *out, double npts,
+                                  cudaStream_t s) {
+    sumsq_final<<<1, 5 * 32, 0, s>>>(work, G, out, npts);
+    return cudaGetLastError();
+}
+
 cudaError_t launch_rms_finish(double *v, double npts, cudaStream_t s) {
     rms_finish<<<1, 32, 0, s>>>(v, npts);
     return cudaGetLastError();

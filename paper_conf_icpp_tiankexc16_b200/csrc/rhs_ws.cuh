@@ -32,6 +32,9 @@
 namespace safara {
 namespace dev {
 
+#ifndef SAFARA_WS_XOREG
+#define SAFARA_WS_XOREG 1  // edge-tile xi case bits in a register (0: recomputed per step, A/B: 4 % slower)
+#endif
 #ifndef SAFARA_WS_SLEEP
 #define SAFARA_WS_SLEEP 20000   // producer waits: suspend-time hint (ns), 0 = plain try_wait
 #endif
@@ -118,7 +121,7 @@ __device__ __forceinline__ void ws_producer(const CUtensorMap *umap, const CUten
     const int warp = (int)threadIdx.x / 32, lane = (int)threadIdx.x % 32;
     uint64_t *full = ws_full(), *afull = ws_afull();
     if (warp == TY) {
-        if (lane != 0) return;
+        if (lane != 0) return;  // (the norm epilogue is entered by rhs_body_ws)
         // in deadline order: step t reads u(t+2) (own column) and f(t)
         for (int s = 0; s < WS_US && s < nu; ++s) ws_issue_u(umap, P, i0, j0, ka + s, s);
         for (int s = 0; s < WS_FS && s < nf; ++s) ws_issue_f(fmap, P, i0, j0, ka + s, s);
@@ -164,16 +167,29 @@ __device__ __forceinline__ void ws_producer(const CUtensorMap *umap, const CUten
 // Consumer per-thread state (as rhs_kernel.cuh Seg, aux from smem).
 struct SegW {
     double *rptr;
-    int uc, ac, fo;
+    int uc, ac;
     bool active, mid_x;
     int ycase;
+#if SAFARA_WS_XOREG
     int xo;
+#endif
     double a[3][5];
     double rq, sq;   // rho_i / square of plane k-1 (planes k, k+1: from the aux ring)
     double tp[5];
+    double ss[5];    // NORM: this thread's sum of rhs_m^2 over its march (f1)
 };
 
-template <int R, bool UD>
+// Edge column tiles: the xi-dissipation case bits and i+-2 redirections of
+// this lane (rhs_kernel.cuh SAFARA_XREG), from blockIdx / laneid.
+__device__ __forceinline__ int ws_xo(const Params &P) {
+    const int col = (int)blockIdx.x % P.ncol;
+    const int i = 1 + (col % P.ntx) * TX + (int)(threadIdx.x % 32);
+    const Cases cs = cases_of(i, P.nx);
+    return (i == P.nx - 3 ? 3 : 2) | ((i == 2 ? 3 : 2) << 8) | (cs.hm1 ? 1 << 16 : 0) |
+           (cs.five ? 1 << 17 : 0) | (cs.hp1 ? 1 << 18 : 0);
+}
+
+template <int R, bool UD, bool AUX, bool NORM>
 __device__ __forceinline__ void ws_step(SegW &g, const Params &P, int k, int q, int ka) {
     constexpr int Q = R % 3, Z = (R + 1) % 3, PI = (R + 2) % 3;  // planes k-1, k, k+1
     const Coef &C = P.c;
@@ -186,7 +202,9 @@ __device__ __forceinline__ void ws_step(SegW &g, const Params &P, int k, int q, 
         mbar_wait(&ws_ffull()[q % WS_FS], (uint32_t)(q / WS_FS) & 1u);
         const double *fs = ws_f() + (size_t)(q % WS_FS) * F_SLOT;
 #pragma unroll
-        for (int m = 0; m < 5; ++m) acc[m] = fs[m * TY * FX + g.fo];
+        // own forcing: (ty, tx+1) of the FX-wide tile = aux-tile index - AXW
+        static_assert(FX == AXW, "forcing and aux tiles share the row width");
+        for (int m = 0; m < 5; ++m) acc[m] = fs[m * TY * FX - AXW + g.ac];
         __syncwarp();
         if ((threadIdx.x & 31) == 0) mbar_arrive(&ws_fempty()[q % WS_FS]);
     }
@@ -207,6 +225,11 @@ __device__ __forceinline__ void ws_step(SegW &g, const Params &P, int k, int q, 
     vc[2] = wz[3] * r0;
     const double qsc = s0 * r0;
     const double pc = wz[4] * r0;
+    if (AUX && g.active) {  // f1: the step-0 fields of this point (plane k)
+        const int kl = k - P.k0;
+        const int off = (int)(g.rptr - P.r) - SK(r) * kl;
+        store_aux(P, off, kl, r0, vc[0], vc[1], vc[2], s0, qsc, wz[4]);
+    }
     auto zeta = [&]() {
         Nb p, qn;
 #pragma unroll
@@ -237,7 +260,11 @@ __device__ __forceinline__ void ws_step(SegW &g, const Params &P, int k, int q, 
                 load5(qq, s, g.uc - 2);
                 diss_terms<false>(t, qq, qn.u, wz, p.u, pp, Cases{});
             } else {
+#if SAFARA_WS_XOREG
                 const int xo = g.xo;
+#else
+                const int xo = ws_xo(P);  // edge tiles only: recomputed, no live register
+#endif
                 load5(pp, s, g.uc + (xo & 0xff));
                 load5(qq, s, g.uc - ((xo >> 8) & 0xff));
                 diss_terms_table(t, qq, qn.u, wz, p.u, pp, (xo & (1 << 16)) ? -4.0 : 0.0,
@@ -291,7 +318,9 @@ __device__ __forceinline__ void ws_step(SegW &g, const Params &P, int k, int q, 
         double *rp = g.rptr;
 #pragma unroll
         for (int m = 0; m < 5; ++m) {
-            __stcs(rp, acc[m] * C.dt);
+            const double v = acc[m] * C.dt;
+            __stcs(rp, v);
+            if (NORM) g.ss[m] = __fma_rn(v, v, g.ss[m]);  // f1: NPB rhs_norm numerator
             rp += SM(r);
         }
     }
@@ -304,28 +333,78 @@ __device__ __forceinline__ void ws_step(SegW &g, const Params &P, int k, int q, 
     (void)ka;
 }
 
-template <bool UD>
+// f1 fused rhs_norm, after the march.  Consumers: warp trees of their
+// per-thread sums into red[warp][m], then arrive on named barrier 2.  The
+// producer warpgroup (idle by then, few registers -- so the consumers' k march
+// keeps its allocation) waits there, forms this CTA's partials (warps in
+// order: deterministic for a given launch) and the last CTA to finish sums
+// every CTA's partials in CTA order and finishes NPB rhs_norm (no second
+// launch), leaving the counter at 0.
+__shared__ double ws_red[TY][5];
+__shared__ int ws_last;
+constexpr int WS_NORM_BAR = 2;
+
+__device__ __forceinline__ void ws_norm_consumer(const double (&ss)[5], int tid) {
+    const int warp = tid / 32, lane = tid % 32;
+#pragma unroll
+    for (int m = 0; m < 5; ++m) {
+        double v = ss[m];
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) v += __shfl_down_sync(0xffffffffu, v, o);
+        if (lane == 0) ws_red[warp][m] = v;
+    }
+    asm volatile("bar.arrive %0, %1;" ::"n"(WS_NORM_BAR), "n"(WS_THREADS) : "memory");
+}
+
+__device__ __forceinline__ void ws_norm_producer(const Params &P) {
+    asm volatile("bar.sync %0, %1;" ::"n"(WS_NORM_BAR), "n"(WS_THREADS) : "memory");
+    const int pt = (int)threadIdx.x - TY * 32;  // 0 .. 127
+    if (pt < 5) {
+        double t = 0.0;
+        for (int w = 0; w < TY; ++w) t += ws_red[w][pt];
+        P.norm_part[pt * P.ncta + (int)blockIdx.x] = t;
+    }
+    asm volatile("bar.sync 3, 128;" ::: "memory");  // producers: partials stored
+    if (pt == 0) {
+        __threadfence();
+        const unsigned long long old = atomicAdd(P.norm_ctr, 1ull);
+        ws_last = old == (unsigned long long)P.ncta - 1;
+    }
+    asm volatile("bar.sync 3, 128;" ::: "memory");
+    if (ws_last && pt < 5) {
+        __threadfence();
+        double t = 0.0;
+        for (int b = 0; b < P.ncta; ++b) t += __ldcg(P.norm_part + pt * P.ncta + b);
+        P.norm_out[pt] = P.norm_npts > 0.0 ? sqrt(t / P.norm_npts) : t;
+    }
+    if (ws_last && pt == 0) *P.norm_ctr = 0ull;
+}
+
+template <bool UD, bool AUX, bool NORM>
 __device__ __forceinline__ void ws_consumer(const Params &P) {
     int col, ka, kb;
     ws_segment(P, col, ka, kb);
-    if (ka >= kb) return;
     const int tid = (int)threadIdx.x;
+    if (ka >= kb) {
+        if (NORM) {  // an empty k-part still reports (zero) to the norm barrier
+            const double z[5] = {0.0, 0.0, 0.0, 0.0, 0.0};
+            ws_norm_consumer(z, tid);
+        }
+        return;
+    }
     const int tx = tid % TX, ty = tid / TX;
     const int i0 = 1 + (col % P.ntx) * TX, j0 = 1 + (col / P.ntx) * TY;
     const int i = i0 + tx, j = j0 + ty;
     const int nx_s = reread(P.nx), ny_s = reread(P.ny);
     SegW g;
     g.active = (i <= nx_s - 2) && (j <= ny_s - 2);
-    g.fo = ty * FX + tx + 1;
     g.uc = (ty + 2) * UX + (tx + HX);
     g.ac = (ty + 1) * AXW + (tx + 1);
     g.mid_x = is_mid(i0, P.nx) && is_mid(i0 + TX - 1, P.nx);
-    {
-        const Cases cs = cases_of(i0 + tx, P.nx);
-        g.xo = (i0 + tx == P.nx - 3 ? 3 : 2) | ((i0 + tx == 2 ? 3 : 2) << 8) |
-               (cs.hm1 ? 1 << 16 : 0) | (cs.five ? 1 << 17 : 0) | (cs.hp1 ? 1 << 18 : 0);
-    }
     g.ycase = is_mid(j, ny_s) ? 0 : j == 1 ? 1 : j == 2 ? 2 : j == ny_s - 3 ? 3 : 4;
+#if SAFARA_WS_XOREG
+    g.xo = ws_xo(P);
+#endif
     g.rptr = P.r + ((idx_t)i + SY(r) * j + SK(r) * (ka - P.k0));
     double *su = ws_u();
     {   // window: planes ka-2, ka-1 from global memory, ka and ka+1 from the ring
@@ -346,17 +425,20 @@ __device__ __forceinline__ void ws_consumer(const Params &P) {
         mbar_wait(&ws_full()[1], 0u);
         load5(g.a[2], su + (size_t)1 * U_SLOT, g.uc);
     }
+#pragma unroll
+    for (int m = 0; m < 5; ++m) g.ss[m] = 0.0;
     int k = ka, q = 0;
 #pragma unroll 1
     for (; k + 3 <= kb; k += 3, q += 3) {
-        ws_step<0, UD>(g, P, k, q, ka);
-        ws_step<1, UD>(g, P, k + 1, q + 1, ka);
-        ws_step<2, UD>(g, P, k + 2, q + 2, ka);
+        ws_step<0, UD, AUX, NORM>(g, P, k, q, ka);
+        ws_step<1, UD, AUX, NORM>(g, P, k + 1, q + 1, ka);
+        ws_step<2, UD, AUX, NORM>(g, P, k + 2, q + 2, ka);
     }
     if (k < kb) {
-        ws_step<0, UD>(g, P, k, q, ka);
-        if (k + 1 < kb) ws_step<1, UD>(g, P, k + 1, q + 1, ka);
+        ws_step<0, UD, AUX, NORM>(g, P, k, q, ka);
+        if (k + 1 < kb) ws_step<1, UD, AUX, NORM>(g, P, k + 1, q + 1, ka);
     }
+    if (NORM) ws_norm_consumer(g.ss, tid);
 }
 
 // SAFARA_TIMELINE builds: {start, end, smid | cycles << 16} of this CTA
@@ -378,7 +460,7 @@ __device__ __forceinline__ void ws_timeline(const Params &P, unsigned long long 
 #endif
 }
 
-template <bool UD>
+template <bool UD, bool AUX, bool NORM>
 __device__ __forceinline__ void rhs_body_ws(const CUtensorMap *umap, const CUtensorMap *fmap,
                                             const Params &P) {
     unsigned long long t_start = 0;
@@ -392,7 +474,7 @@ __device__ __forceinline__ void rhs_body_ws(const CUtensorMap *umap, const CUten
     grid_dep_launch();
     if ((int)blockIdx.x >= P.ncta) {  // the boundary faces (extra CTAs on idle SMs)
         grid_dep_wait();
-        copy_faces<false>(P, (int)blockIdx.x - P.ncta, P.nface_cta);
+        copy_faces<AUX>(P, (int)blockIdx.x - P.ncta, P.nface_cta);
         __syncthreads();
         if (threadIdx.x == 0) ws_timeline(P, t_start, c_start);
         return;
@@ -414,13 +496,14 @@ __device__ __forceinline__ void rhs_body_ws(const CUtensorMap *umap, const CUten
     }
     __syncthreads();
     grid_dep_wait();
-    if (P.nface_cta == 0) copy_faces<false>(P, (int)blockIdx.x, P.ncta);
+    if (P.nface_cta == 0) copy_faces<AUX>(P, (int)blockIdx.x, P.ncta);
     if (tid >= TY * 32) {
         setmaxnreg_dec_producer();
         ws_producer(umap, fmap, P);
+        if (NORM) ws_norm_producer(P);
     } else {
         setmaxnreg_inc_consumer();
-        ws_consumer<UD>(P);
+        ws_consumer<UD, AUX, NORM>(P);
         if (tid == 0) ws_timeline(P, t_start, c_start);
     }
 }

@@ -130,6 +130,10 @@ struct Params {
     unsigned long long *pflags, *pflags_lo, *pflags_hi;
     unsigned long long epoch;  // 0: none; SAFARA_PEER_EPOCH_AUTO: device counter
     unsigned long long peer_timeout_ns;  // bounded flag waits, then __trap()
+    double *norm_part;     // f1 fused rhs_norm: per-CTA partial sums [m * ncta + cta] (NULL: none)
+    unsigned long long *norm_ctr;  // CTAs done (0 between passes; the last CTA resets it)
+    double *norm_out;      // 5 doubles: sqrt(sum / norm_npts), or the sums if norm_npts == 0
+    double norm_npts;
     unsigned long long *dbg;  // SAFARA_TIMELINE builds: per-CTA {start, end, smid}
     unsigned long long *steplog;  // SAFARA_STEPLOG builds: per-CTA globaltimer at each step
     Coef c;
@@ -149,6 +153,10 @@ cudaError_t launch_sumsq(const double *rhs, int nx, int ny, int sy, int sm, int 
                          double *work, double *out, cudaStream_t s, double npts = 0.0);
 // v[m] = sqrt(v[m] / npts), m < 5 (rhs_norm after a cross-slab all-reduce)
 cudaError_t launch_rms_finish(double *v, double npts, cudaStream_t s);
+// f1 fused norm: out[m] = sum over the G per-CTA partials work[m * G + b]
+// (in b order), sqrt(sum / npts) when npts > 0
+cudaError_t launch_partials_final(const double *work, int G, double *out, double npts,
+                                  cudaStream_t s);
 // api.cu: the launch counter behind safara_launch_count
 void count_launches(int n);
 

@@ -377,6 +377,22 @@ def _work_for(r: torch.Tensor, stream) -> torch.Tensor:
     return work
 
 
+# safara_rhs_fused scratch: norm work + 8 words, word 0 a CTA counter that
+# must start at zero (zeros at allocation; the library leaves it zero)
+_fused_work: dict[tuple[int, int], torch.Tensor] = {}
+
+
+def _fused_work_for(r: torch.Tensor, stream) -> torch.Tensor:
+    dev = r.device.index if r.device.index is not None else torch.cuda.current_device()
+    key = (dev, int(_stream_ptr(stream) or 0))
+    work = _fused_work.get(key)
+    if work is None:
+        work = torch.zeros(lib().safara_norm_work_doubles() + 8, dtype=torch.float64,
+                           device=r.device)
+        _fused_work[key] = work
+    return work
+
+
 def rhs_sumsq(r: torch.Tensor, nx: int, nz: int | None = None, k0: int = 0, stream=None,
               out: torch.Tensor | None = None, dims: Dims | None = None) -> torch.Tensor:
     """Per-component sums of rhs^2 over the interior points of the planes
@@ -411,6 +427,38 @@ def rhs_rms(r: torch.Tensor, nx: int, stream=None, out: torch.Tensor | None = No
     check(lib().safara_rhs_rms(r.data_ptr(), ctypes.byref(dims), work.data_ptr(), out.data_ptr(),
                                _stream_ptr(stream)), "safara_rhs_rms")
     return out
+
+
+def rhs_fused(u: torch.Tensor, forcing: torch.Tensor, out: torch.Tensor, nx: int,
+              coeffs: Coeffs, aux: torch.Tensor | None = None, rms: bool | torch.Tensor = True,
+              strict: bool = False, stream=None) -> torch.Tensor | None:
+    """safara_rhs_fused: one pass writing rhs, optionally the aux fields, and
+    (rms=True or a 5-element device tensor) NPB rhs_norm accumulated in the
+    store epilogue.  Returns the rms tensor (or None)."""
+    for t, n in ((u, "u"), (forcing, "forcing"), (out, "out")):
+        _check_field(t, n)
+    nz, ny = _canonical_fields(nx, ((u, "u"), (forcing, "forcing"), (out, "out")))
+    dims = canonical_dims(nx, ny, nz)
+    naux = 0
+    if aux is not None:
+        _check_field(aux, "aux")
+        if aux.dim() != 4 or aux.shape[1] not in (SAFARA_AUX_BT, SAFARA_AUX_SP):
+            raise ValueError(f"aux must be (nz, 6|7, ny, sy), got {tuple(aux.shape)}")
+        _check_shape(aux, (nz, aux.shape[1], ny, pitch(nx)), "aux")
+        naux = int(aux.shape[1])
+    out_rms = None
+    if rms is not False and rms is not None:
+        out_rms = rms if isinstance(rms, torch.Tensor) else torch.empty(
+            5, dtype=torch.float64, device=u.device)
+    work = _fused_work_for(u, stream) if out_rms is not None else None
+    check(lib().safara_rhs_fused(u.data_ptr(), forcing.data_ptr(), out.data_ptr(),
+                                 aux.data_ptr() if aux is not None else None, naux,
+                                 work.data_ptr() if work is not None else None,
+                                 out_rms.data_ptr() if out_rms is not None else None,
+                                 ctypes.byref(dims), ctypes.byref(coeffs),
+                                 SAFARA_FLAG_STRICT if strict else 0, _stream_ptr(stream)),
+          "safara_rhs_fused")
+    return out_rms
 
 
 def rhs_norm(r: torch.Tensor, nx: int, stream=None) -> np.ndarray:

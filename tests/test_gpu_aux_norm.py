@@ -203,3 +203,79 @@ def test_aux_analytic_gas_state(strict):
         assert_tol(g_rhs, o_rhs)
     rho, _, _, _, p = primitives(x, y, z)
     np.testing.assert_allclose(g_aux[..., 6], np.sqrt(GAMMA * p / rho), rtol=1e-13)
+
+
+# ---- round 2: rhs_norm fused into the store epilogue (safara_rhs_fused) ----
+
+@pytest.mark.parametrize("bench,cls", [("BT", "W"), ("BT", "C")])
+@pytest.mark.parametrize("with_aux", [False, True])
+def test_fused_norm_matches_oracle(bench, cls, with_aux):
+    """NPB rhs_norm accumulated in the pass (per-thread sums, CTA partials,
+    one finishing launch) equals the oracle's norm of the oracle's rhs; rhs and
+    aux are unchanged by the fusion (STRICT bitwise)."""
+    inp = nasgen.make_class(bench, cls, seed=1, B=1e-2)
+    nz, ny, nx, _ = inp.u.shape
+    c = sr.coeffs_nas(nx, ny, nz, inp.dt)
+    du, df = sr.pack(inp.u), sr.pack(inp.forcing)
+    dr = torch.full_like(du, float("nan"))
+    da = sr.empty_aux(nx, ny, nz, sr.SAFARA_AUX_BT) if with_aux else None
+    n0 = sr.launch_count()
+    rms = sr.rhs_fused(du, df, dr, nx, c, aux=da, rms=True, strict=True)
+    torch.cuda.synchronize()
+    # class C: the warp-specialised kernel finishes the norm in its last CTA
+    # (one launch); small grids take the two-pass path (3 launches)
+    assert sr.launch_count() - n0 == (1 if cls == "C" else 3)
+    o = oracle.compute_rhs(inp.u, inp.forcing, dt=inp.dt, threads=8)
+    assert np.array_equal(sr.unpack(dr, nx), o)
+    if with_aux:
+        assert np.array_equal(sr.unpack_aux(da, nx), oracle.compute_aux(inp.u, 6, dt=inp.dt))
+    want = np.sqrt(oracle.rhs_sumsq(o) / ((nx - 2) * (ny - 2) * (nz - 2)))
+    np.testing.assert_allclose(rms.cpu().numpy(), want, rtol=1e-13, atol=0)
+    # production: same contract (rhs within c5), norm to 1e-13 of the oracle's
+    rms2 = sr.rhs_fused(du, df, dr, nx, c, aux=da, rms=True)
+    torch.cuda.synchronize()
+    np.testing.assert_allclose(rms2.cpu().numpy(), want, rtol=1e-12, atol=0)
+
+
+def test_fused_norm_general_coefficients_falls_back_to_two_pass():
+    """General (non-NAS) coefficients: no fused-norm kernel instance; the
+    library runs the two-pass norm (3 launches) with the same result."""
+    inp = nasgen.make_class("BT", "W", seed=2)
+    nz, ny, nx, _ = inp.u.shape
+    c = sr.coeffs_nas(nx, ny, nz, inp.dt)
+    c.dxt[2] *= 1.01      # dx3 != dx1: the general-coefficient kernel
+    du, df = sr.pack(inp.u), sr.pack(inp.forcing)
+    dr = torch.empty_like(du)
+    n0 = sr.launch_count()
+    rms = sr.rhs_fused(du, df, dr, nx, c, rms=True, strict=True)
+    torch.cuda.synchronize()
+    assert sr.launch_count() - n0 == 3
+    g = sr.unpack(dr, nx)
+    want = np.sqrt(oracle.rhs_sumsq(g) / ((nx - 2) * (ny - 2) * (nz - 2)))
+    np.testing.assert_allclose(rms.cpu().numpy(), want, rtol=1e-13, atol=0)
+
+
+@pytest.mark.parametrize("p", [2, 3, 8])
+def test_slab_norms_sum_to_full_grid_norm(p):
+    """z-slab partial sums (safara_rhs_sumsq per slab, the numerators the
+    sharded all-reduce adds) give the full-grid rhs_norm to 1e-13."""
+    from paper_conf_icpp_tiankexc16_b200 import dist as sd
+    inp = nasgen.make_class("BT", "A", seed=1, B=1e-2)
+    nz, ny, nx, _ = inp.u.shape
+    c = sr.coeffs_nas(nx, ny, nz, inp.dt)
+    ug, fg = sr.pack(inp.u, device="cpu"), sr.pack(inp.forcing, device="cpu")
+    tot = np.zeros(5)
+    for r in range(p):
+        s = sd.make_slab(ug, fg, nx, r, p, device="cuda")
+        k0, nzl = sd.partition(nz, p)[r]
+        # ghosts from the global field (what the exchange delivers)
+        lo, hi = max(0, k0 - 2), min(nz, k0 + nzl + 2)
+        s.u[lo - (k0 - 2):hi - (k0 - 2)] = ug[lo:hi].cuda()
+        sr.rhs_slab(s.u, s.forcing, s.rhs, nx, nz, k0, c, strict=True)
+        tot += sr.rhs_sumsq(s.rhs, nx, nz=nz, k0=k0).cpu().numpy()
+    torch.cuda.synchronize()
+    du, df = sr.pack(inp.u), sr.pack(inp.forcing)
+    dr = torch.empty_like(du)
+    full = sr.rhs_fused(du, df, dr, nx, c, rms=True, strict=True).cpu().numpy()
+    npts = (nx - 2) * (ny - 2) * (nz - 2)
+    np.testing.assert_allclose(np.sqrt(tot / npts), full, rtol=1e-13, atol=0)
