@@ -36,18 +36,29 @@ import subprocess
 import sys
 import tempfile
 
-# Access latencies in SM cycles (B200/B300 microbenchmarks,
-# /opt/skills/guides/B300_MICROARCH.md: L1 hit 32, L2 hit 234-262, DRAM ~580,
-# LDS 29).  An uncoalesced warp access touches up to 32 sectors instead of the
-# 8 of a coalesced fp64 row, so it costs ~4x the transactions.
-LATENCY = {
-    "register": 0,
-    "shared": 29,
-    "l1": 32,
-    "global_coalesced": 250,
-    "global_uncoalesced": 4 * 250,
-    "dram": 580,
-}
+# Access latencies in SM cycles, measured on the B200 by the [19]-style
+# dependent-chain microbenchmark tools/micro/latency.cu
+# -> profiles/latency_r02.json; the guide's B300 numbers are the fallback.
+# "global_coalesced" is an L2 hit (the halo rows a neighbouring tile fetched),
+# "global_uncoalesced" one warp load touching 32 sectors.
+_FALLBACK_LATENCY = {"register": 8, "shared": 29, "l1": 32, "global_coalesced": 250,
+                     "global_uncoalesced": 1000, "dram": 580}
+
+
+def _measured_latency() -> tuple[dict, str]:
+    p = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "profiles",
+                     "latency_r02.json")
+    try:
+        with open(p) as fh:
+            m = json.load(fh)
+        return {"register": m["register"], "shared": m["shared"], "l1": m["l1"],
+                "global_coalesced": m["l2"], "global_uncoalesced": m["global_uncoalesced"],
+                "dram": m["dram"]}, "measured (profiles/latency_r02.json)"
+    except (OSError, KeyError, ValueError):
+        return dict(_FALLBACK_LATENCY), "fallback (B300 guide)"
+
+
+LATENCY, LATENCY_SOURCE = _measured_latency()
 
 
 @dataclasses.dataclass(frozen=True)
@@ -131,61 +142,199 @@ def ptxas_info(log: str) -> dict:
 # ---------------------------------------------------------------------------
 # The kernel's variant family
 # ---------------------------------------------------------------------------
+GRID_C = 162 ** 3                 # BT class C points (the tuned workload)
+SMSPS = 148 * 4                   # SM sub-partitions (schedulers)
+CLOCK_GHZ = 1.75                  # SM clock under the 1 kW power cap (bench clocks)
+SMEM_CARVEOUTS_KB = (0, 8, 16, 32, 64, 100, 132, 164, 196, 228)
+# Calibration of the two empirical terms (one measurement each):
+ETA = 0.78       # issue efficiency vs the STATIC step body (fit: default variant 134 us)
+GAMMA = 0.25     # share of non-FP64 instructions left exposed (3-4 warps per scheduler)
+T_FACE_92 = 108.0  # us, boundary-face CTAs with a 92 KB L1 (profiles/timeline_ws_r02.txt)
+FACE_EXP = 0.65  # L1 sensitivity of the face CTAs (fit: 142 us at 60 KB, 205 us at 28 KB)
+
+
 @dataclasses.dataclass(frozen=True)
 class Variant:
-    ty: int = 12      # CTA tile rows (threads = 32*ty)
-    stages: int = 4   # TMA ring depth
-    rcp: int = 2      # reciprocal refinement (0: 3 Newton, 1: 2 Newton, 2: cubic)
+    """One point of the kernel family.  ws: where the step-0 fields rho_i /
+    square live -- 0 recomputed per use in registers (round-1 kernel), 1
+    evaluated once per point by a producer warpgroup into a shared-memory
+    ring (rhs_ws.cuh); ring / fring: TMA ring depths (u, forcing); xoreg:
+    edge-tile case bits register-resident; ty: tile rows; strict: the
+    bit-identical contract (no FMA contraction)."""
+    ws: int = 1
+    ring: int = 4
+    fring: int = 2
+    xoreg: int = 1
+    ty: int = 12
+    strict: int = 0
+    rcp: int = 2
 
     @property
     def threads(self) -> int:
-        return 32 * self.ty
+        return 32 * (self.ty + (4 if self.ws else 0))
 
     @property
     def reg_limit(self) -> int:
-        # one CTA per SM (shared memory); 64K registers, allocation granule 8
+        if self.ws:  # consumers after setmaxnreg (producers keep 32)
+            return min(255, ((2048 - 4 * 32) // self.ty) // 8 * 8)
         return min(255, (65536 // self.threads) // 8 * 8)
 
+    @property
+    def smem_bytes(self) -> int:
+        tx, hx = 32, 3
+        ux, uy = tx + 2 * hx, self.ty + 4
+        u_slot = ((ux * uy * 5 * 8 + 127) // 128) * 128
+        f_slot = (((tx + 2) * self.ty * 5 * 8 + 127) // 128) * 128
+        if self.ws:
+            aux = ((self.ring * (tx + 2) * (self.ty + 2) * 16 + 127) // 128) * 128
+            return self.ring * u_slot + aux + self.fring * f_slot + (3 * self.ring + 2 * self.fring) * 8
+        return self.ring * (u_slot + f_slot) + (16 + 3 * tx + tx // 2) * 8
+
+    @property
+    def l1_kb(self) -> int:
+        need = (self.smem_bytes + 1024 + 1023) // 1024  # + 1 KB reserved per CTA
+        carve = next(c for c in SMEM_CARVEOUTS_KB if c >= need) if need <= 228 else 228
+        return 256 - carve
+
     def defines(self) -> list[str]:
-        return [f"-DSAFARA_TY={self.ty}", f"-DSAFARA_STAGES={self.stages}",
-                f"-DSAFARA_RCP={self.rcp}"]
+        d = [f"-DSAFARA_TY={self.ty}", f"-DSAFARA_RCP={self.rcp}"]
+        if self.ws:
+            d += [f"-DSAFARA_WS_US={self.ring}", f"-DSAFARA_WS_FS={self.fring}",
+                  f"-DSAFARA_WS_XOREG={self.xoreg}"]
+        else:
+            d += [f"-DSAFARA_STAGES={self.ring}"]
+        return d
+
+    def env(self) -> dict:
+        return {"SAFARA_WS": str(self.ws)}
+
+    def kernel(self) -> str:
+        v = "strict" if self.strict else "fast"
+        name = f"rhs_kernel_{v}_ws_ud" if self.ws else f"rhs_kernel_{v}_ud"
+        return f"_ZN6safara{len(name)}{name}E14CUtensorMap_stS0_NS_6ParamsE"
 
     def tag(self) -> str:
-        return f"ty{self.ty}_s{self.stages}_r{self.rcp}"
+        t = (f"ws_u{self.ring}f{self.fring}x{self.xoreg}" if self.ws else f"r1_s{self.ring}")
+        t += f"_ty{self.ty}" if self.ty != 12 else ""
+        return t + ("_strict" if self.strict else "")
 
 
 def default_family() -> list[Variant]:
-    return [Variant(ty, st, rcp) for ty in (8, 10, 12) for st in (3, 4) for rcp in (0, 2)]
+    """Aux placement x ring depths x register residency x contract: ten
+    variants (SURVEY §8(f) f3's knobs; tile width is fixed by the warp)."""
+    return [Variant(ws=1, ring=4, fring=2, xoreg=1), Variant(ws=1, ring=4, fring=2, xoreg=0),
+            Variant(ws=1, ring=4, fring=4), Variant(ws=1, ring=5, fring=2),
+            Variant(ws=1, ring=3, fring=2), Variant(ws=0, ring=4), Variant(ws=0, ring=5),
+            Variant(ws=0, ring=4, ty=8), Variant(ws=1, ring=4, fring=2, strict=1),
+            Variant(ws=0, ring=4, strict=1)]
+
+
+_FP64 = ("DFMA", "DMUL", "DADD")
+
+
+def sass_loop_stats(obj: str, fn: str) -> dict | None:
+    """Per-point instruction mix of the kernel's k march, read from the SASS
+    of a compiled variant (the compile feedback, as SAFARA reads ptxas):
+    the largest backward-branch loop that contains FP64 work, 3 steps per
+    body (the register-renaming unroll)."""
+    sass = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "-sass", "-fun", fn, obj],
+                          capture_output=True, text=True).stdout
+    ins = []
+    for line in sass.splitlines():
+        m = re.match(r"\s+/\*([0-9a-f]{4,})\*/\s+(.*?);", line)
+        if m:
+            ins.append((int(m.group(1), 16), m.group(2).strip()))
+    if not ins:
+        return None
+    # out-of-line stubs (mbarrier retry blocks) sit after the last EXIT and
+    # branch back into the body: they are not loops
+    last_exit = max((i for i, (_, t) in enumerate(ins) if "EXIT" in t), default=len(ins) - 1)
+    ins = ins[:last_exit + 1]
+    # the k march: the innermost loop holding at least three steps' FP64 work
+    best = None
+    for a, t in ins:
+        m = re.search(r"BRA(?:\.\w+)? 0x([0-9a-f]+)", t)
+        if m and int(m.group(1), 16) < a:
+            lo = int(m.group(1), 16)
+            body = [x for y, x in ins if lo <= y <= a]
+            nfp = sum(1 for x in body if re.sub(r"^@!?U?P\w+\s+", "", x).split()[0].split(".")[0]
+                      in _FP64)
+            if nfp >= 600 and (best is None or len(body) < len(best)):
+                best = body
+    if best is None:
+        return None
+    ops = [re.sub(r"^@!?U?P\w+\s+", "", x).split()[0].split(".")[0] for x in best]
+    steps = 3
+    return {"fp64": sum(o in _FP64 for o in ops) / steps,
+            "lds": sum(o == "LDS" for o in ops) / steps,
+            "local": sum(o in ("STL", "LDL") for o in ops) / steps,
+            "other": sum(o not in _FP64 for o in ops) / steps,
+            "body_instructions": len(best)}
 
 
 def compile_variant(v: Variant, workdir: str) -> dict:
-    """nvcc the production TU with the variant's defines; ptxas feedback."""
+    """nvcc the variant's translation unit with its defines; ptxas feedback
+    (registers, spill bytes) and the SASS mix of its k march."""
     from . import build as b
-    cmd = [b.NVCC, *b.COMMON, "--fmad=true", "-Xptxas", "-v", *v.defines(), "-c",
-           os.path.join(b.CSRC, "rhs_fast.cu"), "-o", os.path.join(workdir, v.tag() + ".o")]
+    unit = "rhs_strict.cu" if v.strict else "rhs_fast.cu"
+    obj = os.path.join(workdir, v.tag() + ".o")
+    cmd = [b.NVCC, *b.COMMON, "--fmad=false" if v.strict else "--fmad=true", "-Xptxas", "-v",
+           *v.defines(), "-c", os.path.join(b.CSRC, unit), "-o", obj]
     res = subprocess.run(cmd, capture_output=True, text=True)
     if res.returncode != 0:
         return {"variant": v, "error": res.stderr[-400:]}
     info = ptxas_info(res.stdout + res.stderr)
-    prod = next((k for k in info if k.endswith("rhs_kernel_fast_udE14CUtensorMap_stS0_NS_6ParamsE")),
-                None)
-    return {"variant": v, "kernels": info, "prod": info.get(prod)}
+    return {"variant": v, "kernels": info, "prod": info.get(v.kernel()),
+            "sass": sass_loop_stats(obj, v.kernel())}
 
 
-def model_cost(v: Variant, regs: int) -> float:
-    """Relative cycles per grid point of a variant (smaller is better), from
-    the same latency table: the u tile's halo is re-read through L2
-    ((32+6)(ty+4)/(32 ty) per point), latency hidden by the warps resident
-    per SM scheduler (ty/4) and by the ring (stages-2 planes in flight)."""
-    halo = (32 + 6) * (v.ty + 4) / (32 * v.ty)
-    hide = (v.ty / 4) * max(1, v.stages - 2)
-    rcp_fp64 = {0: 6, 1: 4, 2: 3}[v.rcp] * 4  # four reciprocals per point
-    return halo * LATENCY["global_coalesced"] / hide + rcp_fp64 + 300
+def model_cost(v: Variant, regs: int, spill_bytes: int = 0, sass: dict | None = None,
+               latency: dict = LATENCY) -> float:
+    """Predicted BT class C pass time (us) of a variant.
+
+    Compute: the k march issues F FP64 and O other warp-instructions per
+    point (SASS of the variant); the FP64 pipe takes 2 cycles per warp
+    instruction, the scheduler 1 per cycle, so one point costs
+    (max(2F, F+O) + GAMMA*O)/32 scheduler cycles (static counts of the step
+    body: both sides of the edge/mid branches) at the calibrated issue
+    efficiency ETA;
+    spills add their local-memory round trips at the measured L1 latency
+    (ptxas spill bytes / 8 accesses if the SASS has none in the loop).
+    Registers: a variant over its budget cannot launch (infinite cost).
+    Grid: the lockstep schedule's busy SMs (ncol tiles x k-parts) relative to
+    the calibrated 140; TMA lookahead below 2 steps exposes one DRAM latency
+    (measured table) per step of the march.
+    Boundary faces: the face CTAs' strided column gathers are L1-bound:
+    T_FACE_92 * (92 KB / L1 KB)^FACE_EXP (calibrated; the carveout a
+    variant's shared memory leaves decides the L1).  The pass takes the
+    longer of the two."""
+    if regs > v.reg_limit:
+        return float("inf")
+    if sass is None:
+        return float("inf")
+    F, O = sass["fp64"], sass["other"]
+    local = sass["local"] if sass["local"] else spill_bytes / 8 / 3
+    c_issue = (max(2 * F, F + O) + GAMMA * O) / 32.0
+    c_spill = local * latency["l1"] / 32.0
+    t_compute = (GRID_C / SMSPS) * (c_issue / ETA + c_spill) / (CLOCK_GHZ * 1e3)
+    # lockstep grid: ncol column tiles x floor(148 / ncol) k-parts; fewer
+    # busy SMs than the calibrated 12-row shape (140 CTAs) stretch the pass
+    ncol = -(-160 // 32) * -(-160 // v.ty)
+    ctas = ncol * max(1, 148 // ncol) if ncol <= 148 else 148
+    t_compute *= 140.0 / min(ctas, 148)
+    # TMA lookahead: a plane is requested ring-2 steps before its own column
+    # is read; with less than 2 steps one DRAM round trip per step is exposed
+    look = v.ring - 2
+    steps = 160 / max(1, 148 // ncol)
+    t_compute += max(0, 2 - look) * steps * latency["dram"] / (CLOCK_GHZ * 1e3)
+    t_face = T_FACE_92 * (92.0 / max(v.l1_kb, 1)) ** FACE_EXP
+    return max(t_compute, t_face)
 
 
 def tune_variants(family=None, jobs: int = 4) -> list[dict]:
     """Compile the family, apply SAFARA's feasibility rule (no spills, within
-    the register budget of the CTA shape) and rank the survivors."""
+    the register budget of the CTA shape) and rank by the
+    model."""
     family = family or default_family()
     with tempfile.TemporaryDirectory() as wd:
         with cf.ThreadPoolExecutor(jobs) as ex:
@@ -196,24 +345,53 @@ def tune_variants(family=None, jobs: int = 4) -> list[dict]:
         if p is None:
             rows.append({"variant": v.tag(), "error": r.get("error", "no kernel")})
             continue
-        ok = p["spill_st"] == 0 and p["spill_ld"] == 0 and p["regs"] <= v.reg_limit
-        rows.append({"variant": v.tag(), "defines": v.defines(), "regs": p["regs"],
-                     "reg_limit": v.reg_limit, "spill_bytes": p["spill_st"] + p["spill_ld"],
-                     "feasible": ok, "model": round(model_cost(v, p["regs"]), 1)})
-    rows.sort(key=lambda r: (not r.get("feasible", False), r.get("model", 1e9)))
+        spill = p["spill_st"] + p["spill_ld"]
+        ok = spill == 0 and p["regs"] <= v.reg_limit
+        rows.append({"variant": v.tag(), "defines": v.defines(), "env": v.env(),
+                     "strict": v.strict, "regs": p["regs"], "reg_limit": v.reg_limit,
+                     "spill_bytes": spill, "smem_kb": round(v.smem_bytes / 1024, 1),
+                     "l1_kb": v.l1_kb, "sass": r.get("sass"), "feasible": ok,
+                     "model_us": round(model_cost(v, p["regs"], spill, r.get("sass")), 1)})
+    rows.sort(key=lambda r: (not r.get("feasible", False), r.get("model_us", 1e9)))
     return rows
 
 
-def time_variant(tag_defines, steps: int = 100) -> float | None:
+def register_feedback(jobs: int = 2) -> dict:
+    """SAFARA's loop (feedback_loop) run against real compiles of the
+    warp-specialised consumer: the candidate is the edge tiles' xi case
+    bits (reuse: every step of an edge tile; replacing them by a register
+    saves their recomputation, ~10 integer instructions at register
+    latency each).  compile_regs builds the variant and reports the
+    registers the consumer demands (ptxas count + spilled words)."""
+    cand = [Candidate("xi_case_bits", uses=10, space="register", regs=1)]
+    lat = dict(LATENCY)
+    lat["register"] = max(lat["register"], 1)
+
+    def compile_regs(names):
+        v = Variant(ws=1, xoreg=1 if "xi_case_bits" in names else 0)
+        with tempfile.TemporaryDirectory() as wd:
+            r = compile_variant(v, wd)
+        p = r["prod"]
+        return p["regs"] + (p["spill_st"] + p["spill_ld"]) // 4
+
+    limit = Variant(ws=1).reg_limit + 4  # registers + a word of slack
+    chosen, hist = feedback_loop(cand, compile_regs, limit, lat)
+    return {"chosen": [c.name for c in chosen], "history": hist, "limit": limit}
+
+
+def time_variant(v: Variant, steps: int = 200, libdir: str | None = None) -> float | None:
     """Build the full library for a variant and time it with bench.py (GPU)."""
     from . import build as b
-    tag, defines = tag_defines
-    out = os.path.join(b.ROOT, "build", f"libsafara_{tag}.so")
-    b.build(force=True, extra=defines, out=out)
-    env = dict(os.environ, SAFARA_LIB=out)
-    res = subprocess.run([sys.executable, os.path.join(b.ROOT, "bench.py"), "--steps", str(steps),
-                          "--warmup", "10", "--no-cpu-baseline", "--no-other-configs", "--soak-s", "0.3",
-                          "--e2e-steps", "0"], capture_output=True, text=True, env=env)
+    libdir = libdir or os.path.join(b.ROOT, "ablibs")
+    out = os.path.join(libdir, f"tune_{v.tag().replace('_strict', '')}.so")
+    if not os.path.exists(out):
+        b.build(force=True, extra=v.defines(), out=out,
+                objdir=os.path.join(libdir, "obj_tune_" + v.tag()))
+    env = dict(os.environ, SAFARA_LIB=out, **v.env())
+    cmd = [sys.executable, os.path.join(b.ROOT, "bench.py"), "--steps", str(steps),
+           "--warmup", "10", "--no-cpu-baseline", "--no-other-configs", "--soak-s", "0.5",
+           "--e2e-steps", "0"] + (["--strict"] if v.strict else [])
+    res = subprocess.run(cmd, capture_output=True, text=True, env=env)
     try:
         return json.loads(res.stdout.strip().splitlines()[-1])["roofline"]["kernel_ms"] * 1e3
     except Exception:
@@ -222,16 +400,45 @@ def time_variant(tag_defines, steps: int = 100) -> float | None:
 
 def main(argv=None):
     ap = argparse.ArgumentParser(description=__doc__.split("\n\n")[0])
-    ap.add_argument("--time", type=int, default=0, help="time the N best feasible variants (GPU)")
+    ap.add_argument("--build", action="store_true",
+                    help="also build each variant's library into ablibs/ (for --time on a GPU box)")
+    ap.add_argument("--time", type=int, default=0, help="time every variant N times (GPU)")
     ap.add_argument("--jobs", type=int, default=4)
     a = ap.parse_args(argv)
+    print(json.dumps({"latency": LATENCY, "source": LATENCY_SOURCE}))
     rows = tune_variants(jobs=a.jobs)
     for r in rows:
         print(json.dumps(r))
+    print(json.dumps({"register_feedback": register_feedback()}))
+    fam = {v.tag(): v for v in default_family()}
+    if a.build:
+        from . import build as b
+        libdir = os.path.join(b.ROOT, "ablibs")
+        os.makedirs(libdir, exist_ok=True)
+
+        def one(v):
+            out = os.path.join(libdir, f"tune_{v.tag().replace('_strict', '')}.so")
+            if not os.path.exists(out):
+                b.build(force=True, extra=v.defines(), out=out,
+                        objdir=os.path.join(libdir, "obj_tune_" + v.tag()))
+            return out
+        with cf.ThreadPoolExecutor(a.jobs) as ex:
+            list(ex.map(one, [v for v in fam.values() if not v.strict]))
     if a.time:
-        for r in [r for r in rows if r.get("feasible")][:a.time]:
-            us = time_variant((r["variant"], r["defines"]))
-            print(json.dumps({"variant": r["variant"], "kernel_us": us}))
+        meas = {}
+        for rep in range(a.time):
+            for r in rows:
+                if "error" in r:
+                    continue
+                us = time_variant(fam[r["variant"]])
+                meas.setdefault(r["variant"], []).append(us)
+                print(json.dumps({"variant": r["variant"], "rep": rep, "kernel_us": us}),
+                      flush=True)
+        best = {k: min(x for x in t if x) for k, t in meas.items() if any(t)}
+        fastest = min(best, key=best.get)
+        pick = next(r["variant"] for r in rows if r.get("feasible"))
+        print(json.dumps({"model_pick": pick, "fastest_measured": fastest,
+                          "match": pick == fastest, "measured_min_us": best}))
 
 
 if __name__ == "__main__":

@@ -66,17 +66,55 @@ def test_ptxas_parser():
 
 
 def test_variant_register_budget():
-    assert st.Variant(ty=12).reg_limit == 168
-    assert st.Variant(ty=8).reg_limit == 255
-    assert st.Variant(ty=10).reg_limit == 200
+    assert st.Variant(ws=0, ty=12).reg_limit == 168
+    assert st.Variant(ws=0, ty=8).reg_limit == 255
+    assert st.Variant(ws=0, ty=10).reg_limit == 200
+    # warp-specialised: 12 consumer warps share what 4 producer warps at 32
+    # registers leave of the 64K file
+    assert st.Variant(ws=1).reg_limit == 160
+
+
+def test_variant_shared_memory_matches_the_kernel_constants():
+    """safara_internal.h: SMEM_BYTES = 4 slots x (u 24320 + forcing 16384) +
+    1 KB of barriers/table; WS_SMEM_BYTES = u 4 x 24320 + aux 4 x 7616 +
+    forcing 2 x 16384 + 16 barriers -> both leave the 92 KB L1 of a 164 KB
+    carveout; 5-slot rings cross into the 196 / 228 KB carveouts."""
+    assert st.Variant(ws=0, ring=4).smem_bytes == 163840
+    assert st.Variant(ws=1, ring=4, fring=2).smem_bytes == 160640
+    assert st.Variant(ws=0, ring=4).l1_kb == 92 and st.Variant(ws=1).l1_kb == 92
+    assert st.Variant(ws=0, ring=5).l1_kb == 28
+    assert st.Variant(ws=1, ring=4, fring=4).l1_kb == 60
+
+
+def test_latency_table_is_measured():
+    """The L of L x C comes from the B200 microbenchmark."""
+    assert st.LATENCY_SOURCE.startswith("measured")
+    L = st.LATENCY
+    assert L["register"] < L["shared"] < L["l1"] < L["global_coalesced"] < L["dram"]
 
 
 def test_tune_compiles_and_ranks_two_variants():
-    """Real nvcc + ptxas feedback for two variants (cross-compiles, no GPU)."""
-    rows = st.tune_variants([st.Variant(12, 4, 2), st.Variant(8, 4, 2)], jobs=2)
+    """Real nvcc + ptxas + SASS feedback for two variants (cross-compiles, no
+    GPU): both spill-free and within budget; the warp-specialised kernel's
+    k march has fewer FP64 and other instructions per step and ranks first
+    (measured on B200: 134.9 vs 142.2 us, profiles/safara_tune_r02.txt)."""
+    rows = st.tune_variants([st.Variant(ws=1), st.Variant(ws=0)], jobs=2)
     assert len(rows) == 2
     for r in rows:
         assert "error" not in r, r
-        assert r["regs"] <= 255 and r["reg_limit"] in (168, 255)
-    prod = next(r for r in rows if r["variant"] == "ty12_s4_r2")
-    assert prod["feasible"] and prod["spill_bytes"] == 0
+        assert r["feasible"] and r["spill_bytes"] == 0
+        assert r["sass"]["fp64"] > 200 and r["sass"]["local"] == 0
+    assert rows[0]["variant"] == "ws_u4f2x1"
+    ws, r1 = rows
+    assert ws["sass"]["fp64"] < r1["sass"]["fp64"]
+    assert ws["sass"]["body_instructions"] < r1["sass"]["body_instructions"]
+    assert ws["model_us"] < r1["model_us"]
+
+
+def test_model_penalises_small_l1_spills_and_short_rings():
+    sass = {"fp64": 375.0, "other": 268.0, "local": 0.0}
+    base = st.model_cost(st.Variant(ws=1), 128, 0, sass)
+    assert st.model_cost(st.Variant(ws=1, fring=4), 128, 0, sass) > base      # L1 60 KB
+    assert st.model_cost(st.Variant(ws=1, ring=3), 128, 0, sass) > base       # 1 step lookahead
+    assert st.model_cost(st.Variant(ws=1), 128, 0, dict(sass, local=3.0)) > base
+    assert st.model_cost(st.Variant(ws=1), 999, 0, sass) == float("inf")     # over budget
