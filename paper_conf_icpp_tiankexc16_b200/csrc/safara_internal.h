@@ -160,7 +160,8 @@ cudaError_t launch_partials_final(const double *work, int G, double *out, double
 // api.cu: the launch counter behind safara_launch_count
 void count_launches(int n);
 
-// seismic.cu: PAPER.md Fig. 8 dz loop (f4)
+// seismic.cu: PAPER.md Fig. 8 dz loop (f4); the bulk-copy kernel when the
+// rows are 16-byte aligned (SAFARA_SEISMIC_LDG=1 forces the LDG kernel)
 cudaError_t launch_seismic_dz(const double *vz1, const double *vz2, const double *vz3, double *out,
                               int nx, int ny, int nz, int sy, int sk, double h, int sms,
                               cudaStream_t s);
