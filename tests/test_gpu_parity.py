@@ -262,6 +262,23 @@ def test_analytic_navier_stokes_field(shape):
     assert_tol(gpu_rhs(u, f, 1e-3, strict=False), o)
 
 
+@pytest.mark.xfail(strict=True, reason="production variant on the cancellation-dominated "
+                   "P7 state (zero forcing, dt = 1): the elementwise c5 bound is missed by up "
+                   "to ~35x at near-zero outputs (DESIGN.md c5; the normwise bound holds)")
+def test_analytic_state_production_elementwise_gap():
+    """Records the gap the header states (include/safara.h, safara_rhs): on
+    O(1e3) terms cancelling to O(1), production is held to the normwise bound
+    only.  Strict xfail: if a change closes the gap, this test says so."""
+    from test_oracle_euler_pins import conservative
+    nz, ny, nx = 49, 49, 49
+    z, y, x = np.meshgrid(np.linspace(0, 1, nz), np.linspace(0, 1, ny),
+                          np.linspace(0, 1, nx), indexing="ij")
+    u = conservative(x, y, z)
+    f = np.zeros_like(u)
+    o = oracle.compute_rhs(u, f, dt=1.0, threads=8)
+    assert_tol(gpu_rhs(u, f, 1.0, strict=False), o)
+
+
 _WS_SCRIPT = r"""
 import sys, numpy as np, torch
 sys.path.insert(0, {root!r})
