@@ -345,7 +345,8 @@ int launch(const double *u, const double *f, double *r, const safara_dims_t &d, 
     // the warp-specialised kernel serves launches whose CTAs each own one
     // (column tile, k range) segment: lockstep over a single plane range,
     // without the f1 aux output or the f2 peer halo
-    const bool ws = g_tune.ws && lockstep && p.parts > 0 && p.n0 == p.nplanes && !peer;
+    const bool ws = g_tune.ws && lockstep && p.parts > 0 && p.n0 == p.nplanes &&
+                    !(peer && aux);
     // f1 fused rhs_norm: the warp-specialised kernel with NAS coefficients
     // writes per-CTA partial sums; otherwise the caller runs the two-pass norm
     if (fused) *fused = norm_work != nullptr && ws && ud;

@@ -69,6 +69,10 @@ __device__ __forceinline__ void ws_issue_u(const CUtensorMap *umap, const Params
     const int c2 = P.pos_j == 2 ? jc : (P.pos_m == 2 ? 0 : kb);
     const int c3 = P.pos_j == 3 ? jc : (P.pos_m == 3 ? 0 : kb);
     uint64_t *bar = &ws_full()[slot];
+    if (k >= P.pk_hi) {  // f2: a neighbour's plane (own column read by peer_col)
+        mbar_arrive(bar);
+        return;
+    }
     mbar_expect_tx(bar, TMA_BYTES);
     tma_load_4d(ws_u() + (size_t)slot * U_SLOT, umap, bar, i0 - HX, c1, c2, c3);
 }
@@ -149,10 +153,11 @@ __device__ __forceinline__ void ws_producer(const CUtensorMap *umap, const CUten
     for (int s = 0; s < nu; ++s) {
         const int slot = s % WS_US;
         ws_pwait(&full[slot], (uint32_t)(s / WS_US) & 1u);
-        // rho_i, square of every point of the tile + halo 1 (App. A step 0)
+        // rho_i, square of every point of the tile + halo 1 (App. A step 0);
+        // none for a neighbour's plane (f2: no tile was loaded)
         const double *ut = ws_u() + (size_t)slot * U_SLOT;
         double2 *at = ax + (size_t)slot * A_SLOT;
-        for (int p = pt; p < A_SLOT; p += WS_AW * 32) {
+        for (int p = ka + s < P.pk_hi ? pt : A_SLOT; p < A_SLOT; p += WS_AW * 32) {
             const int r = p / AXW, c = p - r * AXW;
             const int ui = (r + 1) * UX + (c + HX - 1);
             double rho, sq;
@@ -174,6 +179,7 @@ struct SegW {
     int xo;
 #endif
     double a[3][5];
+    int colo;        // f2 (PEER): own column offset i + sy*j for the neighbours' planes
     double rq, sq;   // rho_i / square of plane k-1 (planes k, k+1: from the aux ring)
     double tp[5];
     double ss[5];    // NORM: this thread's sum of rhs_m^2 over its march (f1)
@@ -189,7 +195,7 @@ __device__ __forceinline__ int ws_xo(const Params &P) {
            (cs.five ? 1 << 17 : 0) | (cs.hp1 ? 1 << 18 : 0);
 }
 
-template <int R, bool UD, bool AUX, bool NORM>
+template <int R, bool UD, bool AUX, bool NORM, bool PEER>
 __device__ __forceinline__ void ws_step(SegW &g, const Params &P, int k, int q, int ka) {
     constexpr int Q = R % 3, Z = (R + 1) % 3, PI = (R + 2) % 3;  // planes k-1, k, k+1
     const Coef &C = P.c;
@@ -237,8 +243,12 @@ __device__ __forceinline__ void ws_step(SegW &g, const Params &P, int k, int q, 
             p.u[m] = g.a[PI][m];
             qn.u[m] = g.a[Q][m];
         }
-        const double2 o1 = ax[(size_t)((q + 1) % WS_US) * A_SLOT + g.ac];  // plane k+1
-        p.rho = o1.x; p.sq = o1.y;
+        if (PEER && k + 1 >= P.pk_hi) {  // f2: plane k+1 is the upper neighbour's
+            aux_of(p.u[0], p.u[1], p.u[2], p.u[3], p.rho, p.sq);
+        } else {
+            const double2 o1 = ax[(size_t)((q + 1) % WS_US) * A_SLOT + g.ac];  // plane k+1
+            p.rho = o1.x; p.sq = o1.y;
+        }
         qn.rho = g.rq; qn.sq = g.sq;
         flux_dir<3, false, UD>(acc, wz, vc, qsc, pc, p, qn, C, 2);
     };
@@ -297,7 +307,10 @@ __device__ __forceinline__ void ws_step(SegW &g, const Params &P, int k, int q, 
 #if !SAFARA_ZETA_FIRST
     zeta();
 #endif
-    load5(an, s2, g.uc);
+    if (PEER && k + 2 >= P.pk_hi)
+        peer_col(an, P, k + 2, g.colo);  // f2: the upper neighbour's own column
+    else
+        load5(an, s2, g.uc);
     {
         double t_z[5];
         if (is_mid(k, P.nz)) {
@@ -380,7 +393,7 @@ __device__ __forceinline__ void ws_norm_producer(const Params &P) {
     if (ws_last && pt == 0) *P.norm_ctr = 0ull;
 }
 
-template <bool UD, bool AUX, bool NORM>
+template <bool UD, bool AUX, bool NORM, bool PEER>
 __device__ __forceinline__ void ws_consumer(const Params &P) {
     int col, ka, kb;
     ws_segment(P, col, ka, kb);
@@ -411,32 +424,45 @@ __device__ __forceinline__ void ws_consumer(const Params &P) {
         const int ic = min(i, nx_s - 1), jc = min(j, ny_s - 1);
         const int lk = ka - P.k0 + P.ukoff;
         const double *uc0 = P.u + (idx_t)(ic + SY(u) * jc);
+        const int colo = ic + P.sy * jc;
+        g.colo = colo;
+        if (ka - 1 < P.pk_lo) {  // f2: planes below the slab are the lower neighbour's
+            peer_col(g.a[0], P, ka - 1, colo);
+        } else {
 #pragma unroll
-        for (int m = 0; m < 5; ++m)
-            g.a[0][m] = lk - 1 >= 0 ? __ldg(uc0 + SM(u) * m + SK(u) * (lk - 1)) : 0.0;
+            for (int m = 0; m < 5; ++m)
+                g.a[0][m] = lk - 1 >= 0 ? __ldg(uc0 + SM(u) * m + SK(u) * (lk - 1)) : 0.0;
+        }
         double am2[5];
+        if (ka - 2 < P.pk_lo) {
+            peer_col(am2, P, ka - 2, colo);
+        } else {
 #pragma unroll
-        for (int m = 0; m < 5; ++m)
-            am2[m] = lk - 2 >= 0 ? __ldg(uc0 + SM(u) * m + SK(u) * (lk - 2)) : 0.0;
+            for (int m = 0; m < 5; ++m)
+                am2[m] = lk - 2 >= 0 ? __ldg(uc0 + SM(u) * m + SK(u) * (lk - 2)) : 0.0;
+        }
         aux_of(g.a[0][0], g.a[0][1], g.a[0][2], g.a[0][3], g.rq, g.sq);
         mbar_wait(&ws_afull()[0], 0u);
         load5(g.a[1], su, g.uc);
         zeta_partial(g.tp, am2, g.a[0], g.a[1], ka, P.nz, is_mid(ka, P.nz));
         mbar_wait(&ws_full()[1], 0u);
-        load5(g.a[2], su + (size_t)1 * U_SLOT, g.uc);
+        if (PEER && ka + 1 >= P.pk_hi)
+            peer_col(g.a[2], P, ka + 1, colo);
+        else
+            load5(g.a[2], su + (size_t)1 * U_SLOT, g.uc);
     }
 #pragma unroll
     for (int m = 0; m < 5; ++m) g.ss[m] = 0.0;
     int k = ka, q = 0;
 #pragma unroll 1
     for (; k + 3 <= kb; k += 3, q += 3) {
-        ws_step<0, UD, AUX, NORM>(g, P, k, q, ka);
-        ws_step<1, UD, AUX, NORM>(g, P, k + 1, q + 1, ka);
-        ws_step<2, UD, AUX, NORM>(g, P, k + 2, q + 2, ka);
+        ws_step<0, UD, AUX, NORM, PEER>(g, P, k, q, ka);
+        ws_step<1, UD, AUX, NORM, PEER>(g, P, k + 1, q + 1, ka);
+        ws_step<2, UD, AUX, NORM, PEER>(g, P, k + 2, q + 2, ka);
     }
     if (k < kb) {
-        ws_step<0, UD, AUX, NORM>(g, P, k, q, ka);
-        if (k + 1 < kb) ws_step<1, UD, AUX, NORM>(g, P, k + 1, q + 1, ka);
+        ws_step<0, UD, AUX, NORM, PEER>(g, P, k, q, ka);
+        if (k + 1 < kb) ws_step<1, UD, AUX, NORM, PEER>(g, P, k + 1, q + 1, ka);
     }
     if (NORM) ws_norm_consumer(g.ss, tid);
 }
@@ -460,7 +486,7 @@ __device__ __forceinline__ void ws_timeline(const Params &P, unsigned long long 
 #endif
 }
 
-template <bool UD, bool AUX, bool NORM>
+template <bool UD, bool AUX, bool NORM, bool PEER>
 __device__ __forceinline__ void rhs_body_ws(const CUtensorMap *umap, const CUtensorMap *fmap,
                                             const Params &P) {
     unsigned long long t_start = 0;
@@ -472,11 +498,18 @@ __device__ __forceinline__ void rhs_body_ws(const CUtensorMap *umap, const CUten
     // PDL (SAFARA_PDL builds): the next pass on the stream may be scheduled
     // now; every global access below waits for the previous grid.
     grid_dep_launch();
+    if (P.epoch) {  // f2: every CTA publishes "my u of this epoch is final"
+        grid_dep_wait();
+        peer_epoch_init(P);
+        __syncthreads();
+        peer_publish(P);
+    }
     if ((int)blockIdx.x >= P.ncta) {  // the boundary faces (extra CTAs on idle SMs)
         grid_dep_wait();
         copy_faces<AUX>(P, (int)blockIdx.x - P.ncta, P.nface_cta);
         __syncthreads();
         if (threadIdx.x == 0) ws_timeline(P, t_start, c_start);
+        peer_arrive(P);
         return;
     }
     const int tid = (int)threadIdx.x;
@@ -503,9 +536,12 @@ __device__ __forceinline__ void rhs_body_ws(const CUtensorMap *umap, const CUten
         if (NORM) ws_norm_producer(P);
     } else {
         setmaxnreg_inc_consumer();
-        ws_consumer<UD, AUX, NORM>(P);
+        ws_consumer<UD, AUX, NORM, PEER>(P);
         if (tid == 0) ws_timeline(P, t_start, c_start);
     }
+    // f2: the grid completes only when no neighbour still reads our u (both
+    // roles meet here; the peer loads were the consumers')
+    peer_arrive(P);
 }
 
 }  // namespace dev

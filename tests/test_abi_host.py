@@ -39,10 +39,21 @@ def test_sass_is_sm100a_with_tma():
 
 
 def test_ptxas_zero_spills():
-    build.build(force=True)
-    log = open(build.os.path.join(build.BUILD, "ptxas.txt")).read()
-    assert log.count("0 bytes spill stores, 0 bytes spill loads") >= 2, log
-    assert "0 bytes stack frame" in log
+    """ptxas -v of the current build: the production kernels (the round-2
+    warp-specialised NAS instance the bench runs, its aux variant, and the
+    round-1 production kernel) have no stack frame and no spill bytes."""
+    from paper_conf_icpp_tiankexc16_b200 import safara_tune as st
+    build.build()
+    path = build.os.path.join(build.BUILD, "ptxas.txt")
+    if not build.os.path.exists(path):
+        build.build(force=True)
+    info = st.ptxas_info(open(path).read())
+    for name in ("rhs_kernel_fast_ws_ud", "rhs_kernel_fast_ws_ud_aux", "rhs_kernel_fast_ud",
+                 "rhs_kernel_fast_ud_aux"):
+        key = f"_ZN6safara{len(name)}{name}E14CUtensorMap_stS0_NS_6ParamsE"
+        assert key in info, name
+        k = info[key]
+        assert k["spill_st"] == 0 and k["spill_ld"] == 0 and k["stack"] == 0, (name, k)
 
 
 def test_pitch_and_canonical_dims(L):
