@@ -271,7 +271,11 @@ int launch(const double *u, const double *f, double *r, const safara_dims_t &d, 
     // CTA takes a share before its march
     const long long face_pts =
         (long long)(2 * d.nx + 2 * (d.ny - 2)) * (fk_hi - fk_lo) + 2LL * (d.nx - 2) * (d.ny - 2);
-    p.nface_cta = (g_tune.face_ctas && !aux && fk_hi > fk_lo && p.units > 0 && ncta < max_ctas)
+    if (g_tune.face_ctas < 0) {  // PROBE ONLY (SAFARA_FACE_CTAS=-1): boundary faces skipped
+        p.fk_lo = p.fk_hi = 0;
+        fk_lo = fk_hi = 0;
+    }
+    p.nface_cta = (g_tune.face_ctas > 0 && !aux && fk_hi > fk_lo && p.units > 0 && ncta < max_ctas)
                       ? (int)std::min<long long>({max_ctas - ncta, 32, (face_pts + 4095) / 4096})
                       : 0;
 
@@ -347,6 +351,7 @@ int launch(const double *u, const double *f, double *r, const safara_dims_t &d, 
     // without the f1 aux output or the f2 peer halo
     const bool ws = g_tune.ws && lockstep && p.parts > 0 && p.n0 == p.nplanes &&
                     !(peer && aux);
+
     // f1 fused rhs_norm: the warp-specialised kernel with NAS coefficients
     // writes per-CTA partial sums; otherwise the caller runs the two-pass norm
     if (fused) *fused = norm_work != nullptr && ws && ud;
