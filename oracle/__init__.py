@@ -10,8 +10,10 @@ Arrays cross this wrapper in the *logical* layout ``(nz, ny, nx, 5)`` float64
 (C order, component fastest), the layout ``nasgen`` produces; the wrapper pads
 to the NAS-BT layout ``u[nz][ny'][nx'][5]`` the C code uses.
 
-Pins: see ``tests/test_oracle_pins.py`` (P1-P6).  The NAS
-constants vs the NPB source are "parity unpinned" (reading c2).
+Pins: see ``tests/test_oracle_pins.py`` (P1-P6), ``test_oracle_exact_pins.py``
+(P3), ``test_oracle_euler_pins.py`` (P7) and ``test_oracle_bt_pins.py`` (P8:
+the full BT step reproduces NPB's class S/W/A verification norms, pinning the
+NAS constants against NPB itself, reading c2).
 """
 from __future__ import annotations
 

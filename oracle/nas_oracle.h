@@ -23,9 +23,11 @@
  * closed forms (dissipation operator = B^T B), P5 forcing affinity, P6 i<->j
  * symmetry, P7 O(h^2) convergence to the compressible Navier-Stokes operator
  * (tests/test_oracle_euler_pins.py: pins c1, c2, t?2 and the viscous /
- * artificial-dissipation constant combinations).  The physical parameter
- * values (gamma, mu, Pr, dx..dz, dssp) vs the NPB source: parity unpinned
- * (reading c2).
+ * artificial-dissipation constant combinations), P8 NPB verification
+ * (tests/test_oracle_bt_pins.py): the full BT time step of nas_bt.c from NPB's
+ * initialize reproduces NPB BT's own class S/W/A verification norms to
+ * <= 1e-12 (NPB accepts 1e-8), which pins the physical parameter values
+ * (gamma, mu, Pr, dx..dz, dssp) against NPB itself (reading c2).
  */
 #ifndef NAS_ORACLE_H
 #define NAS_ORACLE_H

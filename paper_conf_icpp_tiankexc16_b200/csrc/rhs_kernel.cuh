@@ -566,7 +566,11 @@ __device__ __forceinline__ void diss_apply(double (&acc)[5], const double (&t)[5
 template <bool AUX>
 __device__ __forceinline__ void copy_faces(const Params &P, int cta, int nctas) {
     const int nx = P.nx, ny = P.ny;
+#ifdef SAFARA_PROBE_NO_IFACE
+    const int per = 2 * nx;  // timing probe only: i-faces skipped
+#else
     const int per = 2 * nx + 2 * (ny - 2);
+#endif
     const int nloc = P.fk_hi - P.fk_lo;
     if (nloc <= 0) return;
     const long long nper = (long long)per * nloc;
