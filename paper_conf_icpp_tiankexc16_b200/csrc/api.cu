@@ -611,9 +611,15 @@ int safara_ipc_get(const void *dptr, void *handle, int64_t *offset) {
     }
     CUdeviceptr base = 0;
     size_t size = 0;
-    if (range(&base, &size, (CUdeviceptr)dptr) != CUDA_SUCCESS) return SAFARA_ERR_CUDA;
+    if (range(&base, &size, (CUdeviceptr)dptr) != CUDA_SUCCESS) {
+        (void)cudaGetLastError();
+        return SAFARA_ERR_CUDA;
+    }
     cudaIpcMemHandle_t h;
-    if (cudaIpcGetMemHandle(&h, (void *)base) != cudaSuccess) return SAFARA_ERR_CUDA;
+    if (cudaIpcGetMemHandle(&h, (void *)base) != cudaSuccess) {
+        (void)cudaGetLastError();  // not sticky: do not leave it for a later call to report
+        return SAFARA_ERR_CUDA;
+    }
     static_assert(sizeof(h) == SAFARA_IPC_HANDLE_BYTES, "IPC handle size");
     std::memcpy(handle, &h, sizeof(h));
     *offset = (int64_t)((CUdeviceptr)dptr - base);
@@ -625,8 +631,10 @@ int safara_ipc_open(const void *handle, int64_t offset, void **dptr) {
     cudaIpcMemHandle_t h;
     std::memcpy(&h, handle, sizeof(h));
     void *base = nullptr;
-    if (cudaIpcOpenMemHandle(&base, h, cudaIpcMemLazyEnablePeerAccess) != cudaSuccess)
+    if (cudaIpcOpenMemHandle(&base, h, cudaIpcMemLazyEnablePeerAccess) != cudaSuccess) {
+        (void)cudaGetLastError();
         return SAFARA_ERR_CUDA;
+    }
     *dptr = (char *)base + offset;
     return SAFARA_OK;
 }
