@@ -561,6 +561,22 @@ __device__ __forceinline__ void diss_apply(double (&acc)[5], const double (&t)[5
     for (int m = 0; m < 5; ++m) acc[m] = acc[m] - dssp * t[m];
 }
 
+// Face copy cache policy (experiments: SAFARA_FACE_CACHE 0 streaming .cs
+// loads/stores, 1 .cg loads (L2 only) + .cs stores, 2 .cg loads + .cg stores)
+#ifndef SAFARA_FACE_CACHE
+#define SAFARA_FACE_CACHE 2
+#endif
+#if SAFARA_FACE_CACHE == 0
+#define FACE_LD __ldcs
+#define FACE_ST __stcs
+#elif SAFARA_FACE_CACHE == 1
+#define FACE_LD __ldcg
+#define FACE_ST __stcs
+#else
+#define FACE_LD __ldcg
+#define FACE_ST __stcg
+#endif
+
 // Copy forcing -> rhs on this launch's boundary-face points (rhs = forcing,
 // unscaled; App. A step 1, reading c3), spread over all CTAs.
 template <bool AUX>
@@ -618,7 +634,7 @@ __device__ __forceinline__ void copy_faces(const Params &P, int cta, int nctas) 
                 }
                 off[b] = i + SY(f) * j + SK(f) * kl;
 #pragma unroll
-                for (int m = 0; m < 5; ++m) v[b][m] = __ldcs(P.f + off[b] + SM(f) * m);
+                for (int m = 0; m < 5; ++m) v[b][m] = FACE_LD(P.f + off[b] + SM(f) * m);
                 if (AUX) {  // aux of the face point from u (u plane = kl + ukoff)
                     const double *up = P.u + (i + SY(u) * j + SK(u) * (kl + P.ukoff));
                     const double u1 = __ldg(up), u2 = __ldg(up + SM(u)), u3 = __ldg(up + 2 * SM(u));
@@ -634,7 +650,7 @@ __device__ __forceinline__ void copy_faces(const Params &P, int cta, int nctas) 
         for (int b = 0; b < FB; ++b)
             if (off[b] >= 0) {
 #pragma unroll
-                for (int m = 0; m < 5; ++m) __stcs(P.r + off[b] + SM(r) * m, v[b][m]);
+                for (int m = 0; m < 5; ++m) FACE_ST(P.r + off[b] + SM(r) * m, v[b][m]);
             }
     }
 }
