@@ -44,7 +44,8 @@ def parse():
     ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--e2e-chunks", type=int, default=8,
                     help="k-chunks of the pipelined H2D / compute / D2H e2e path")
-    ap.add_argument("--workload", default="rhs", choices=["rhs", "rhs_aux", "rhs_norm", "rhs_aux_norm", "seismic_dz"],
+    ap.add_argument("--workload", default="rhs", choices=["rhs", "rhs_aux", "rhs_norm", "rhs_aux_norm", "seismic_dz",
+                                             "bt_step"],
                     help="rhs: the headline compute_rhs pass; rhs_aux: the same pass also "
                          "writing the 6 step-0 fields (SURVEY §8(f) f1); seismic_dz: the "
                          "PAPER.md Fig. 8 loop (f4) on --seismic-n^3")
@@ -466,6 +467,51 @@ def run_single(args):
     print(json.dumps(line), flush=True)
 
 
+def run_bt_step(args):
+    """one whole NPB BT time step per step (safara_bt_step:
+    compute_rhs with the aux fields, x/y/z block-tridiagonal line solves, add;
+    5 launches) at the class of --config (BT-C by default), from NPB's
+    initialize with exact_rhs forcing; reported in grid-points/s of steps.
+    The line solves are a plain one-thread-per-line kernel (not the tuned
+    path); this line measures the whole step, not a roofline claim."""
+    import torch
+
+    import nasgen
+    import paper_conf_icpp_tiankexc16_b200 as sr
+
+    torch.cuda.set_device(0)
+    sr.init(0)
+    bench, cls, n, dt = config_of(args)
+    u0 = nasgen.nas_initialize(n, n, n)
+    f = nasgen.exact_rhs(n, n, n, dt)
+    st = sr.BtState(sr.pack(u0), sr.pack(f), n, dt)
+    stream = torch.cuda.current_stream()
+    for _ in range(max(args.warmup, 3)):
+        st.step(strict=args.strict)
+    torch.cuda.synchronize()
+    sampler = ClockSampler(0)
+    sampler.start()
+    l0 = sr.launch_count()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for _ in range(args.steps):
+        st.step(strict=args.strict)
+    e1.record(stream)
+    torch.cuda.synchronize()
+    clocks = ClockSampler.summarise(sampler.stop())
+    ms = e0.elapsed_time(e1) / args.steps
+    pts = n ** 3
+    print(json.dumps({
+        "metric": "BT time steps x grid-points/s", "value": pts / (ms * 1e-3) / 1e9,
+        "unit": "Gpt/s", "n_gpus": 1, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": ms, "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+        "dtype": "f64", "data": "synthetic (NPB initialize + exact_rhs)",
+        "config": {"workload": f"NPB BT time step class {cls} {n}^3 fp64 (f4(ii))",
+                   "grid": [n, n, n], "points": pts,
+                   "variant": "strict" if args.strict else "production"},
+        "clocks": clocks, "gpu_launches": sr.launch_count() - l0}), flush=True)
+
+
 def run_seismic(args):
     """PAPER.md Fig. 8 dz loop: 3 inputs + 1 output of
     n^3 doubles, 32 algorithmic bytes per point (HBM-bound)."""
@@ -595,6 +641,9 @@ def main():
         args.graph = 20 if multi and args.halo == "peer" else 0
     if args.slab_sim:
         run_slab_sim(args)
+        return
+    if args.workload == "bt_step" and args.impl != "reference":
+        run_bt_step(args)
         return
     if args.workload == "seismic_dz" and args.impl != "reference":
         run_seismic(args)
