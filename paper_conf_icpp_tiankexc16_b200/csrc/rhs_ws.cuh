@@ -45,6 +45,22 @@ __device__ __forceinline__ void ws_pwait(uint64_t *bar, uint32_t parity) {
     mbar_wait(bar, parity);
 #endif
 }
+#ifndef SAFARA_WS_PROBE
+#define SAFARA_WS_PROBE 0  // timing probes (wrong rhs): 1 no zeta dissipation, 2 no xi dissipation (mid tiles)
+#endif
+#ifndef SAFARA_WS_CSLEEP
+#define SAFARA_WS_CSLEEP 0      // consumer waits: suspend-time hint (ns), 0 = plain try_wait spin
+#endif
+#ifndef SAFARA_WS_STORE
+#define SAFARA_WS_STORE 0       // rhs stores: 0 st.global.cs, 1 default policy
+#endif
+__device__ __forceinline__ void ws_cwait(uint64_t *bar, uint32_t parity) {
+#if SAFARA_WS_CSLEEP > 0
+    mbar_wait_sleep(bar, parity, SAFARA_WS_CSLEEP);
+#else
+    mbar_wait(bar, parity);
+#endif
+}
 __device__ __forceinline__ double *ws_u() { return reinterpret_cast<double *>(smem_raw); }
 __device__ __forceinline__ double2 *ws_aux() {
     return reinterpret_cast<double2 *>(smem_raw + WS_U_BYTES);
@@ -195,7 +211,50 @@ __device__ __forceinline__ int ws_xo(const Params &P) {
            (cs.five ? 1 << 17 : 0) | (cs.hp1 ? 1 << 18 : 0);
 }
 
-template <int R, bool UD, bool AUX, bool NORM, bool PEER>
+// FAST steps (interior planes: k and k+1 take the mid zeta cases, no peer
+// plane involved): every wait at the top and then ONE branch-free basic
+// block -- xi dissipation in the per-lane table form for every tile, eta in
+// a per-warp coefficient form for every row, predicated stores -- so the
+// scheduler can overlap the shared-memory loads of all three directions with
+// the FP64 work (the generic step is ~8 basic blocks, several of them "load,
+// then use at once").  Bitwise identical to the generic step (see
+// diss_eta_coef).
+#ifndef SAFARA_WS_FAST
+#define SAFARA_WS_FAST 0  // A/B on B200: 1 % slower (profiles/ab_fast_r02.txt)
+#endif
+// eta dissipation weights {c-2, c-1, c0, c+1, c+2} of the NAS cases
+// (0 interior, 1 j=1, 2 j=2, 3 j=ny-3, 4 j=ny-2): t = c-2*a-2, then
+// fma(c-1, a-1, t), + c0*a0, fma(c+1, a+1, t), fma(c+2, a+2, t).  A zero
+// weight multiplies a finite value (exact 0 / t + 0 = t) and unit / -4 / 6 /
+// 5 products are the NAS ones, so every case rounds exactly as the NAS text
+// (diss_terms_case) in STRICT; the production build contracts the same way
+// as the interior form.
+__constant__ double c_eta_coef[5][5] = {{1.0, -4.0, 6.0, -4.0, 1.0},
+                                         {0.0, 0.0, 5.0, -4.0, 1.0},
+                                         {0.0, -4.0, 6.0, -4.0, 1.0},
+                                         {1.0, -4.0, 6.0, -4.0, 0.0},
+                                         {1.0, -4.0, 5.0, 0.0, 0.0}};
+__device__ __forceinline__ void diss_eta_coef(double (&t)[5], const double (&am2)[5],
+                                              const double (&am1)[5], const double (&a0)[5],
+                                              const double (&ap1)[5], const double (&ap2)[5],
+                                              const double *ce) {
+    const double cm2 = ce[0], cm1 = ce[1], cc = ce[2], cp1 = ce[3], cp2 = ce[4];
+#pragma unroll
+    for (int m = 0; m < 5; ++m) {
+        double x = cm2 * am2[m];
+        x = __fma_rn(cm1, am1[m], x);
+        x = x + cc * a0[m];
+        x = __fma_rn(cp1, ap1[m], x);
+        t[m] = __fma_rn(cp2, ap2[m], x);
+    }
+}
+__device__ __forceinline__ void st_cs_pred(double *p, double v, bool pred) {
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q st.global.cs.f64 [%0], %1;\n\t}" ::"l"(p),
+                 "d"(v), "r"((unsigned)pred)
+                 : "memory");
+}
+
+template <int R, bool UD, bool AUX, bool NORM, bool PEER, bool FAST = false>
 __device__ __forceinline__ void ws_step(SegW &g, const Params &P, int k, int q, int ka) {
     constexpr int Q = R % 3, Z = (R + 1) % 3, PI = (R + 2) % 3;  // planes k-1, k, k+1
     const Coef &C = P.c;
@@ -204,8 +263,13 @@ __device__ __forceinline__ void ws_step(SegW &g, const Params &P, int k, int q, 
     const double *s = su + (size_t)(q % WS_US) * U_SLOT;
     const double2 *a0 = ax + (size_t)(q % WS_US) * A_SLOT;
     double acc[5];
+    if (FAST) {  // every wait of the step first
+        ws_cwait(&ws_ffull()[q % WS_FS], (uint32_t)(q / WS_FS) & 1u);
+        ws_cwait(&ws_afull()[(q + 1) % WS_US], (uint32_t)((q + 1) / WS_US) & 1u);
+        ws_cwait(&ws_full()[(q + 2) % WS_US], (uint32_t)((q + 2) / WS_US) & 1u);
+    }
     {   // forcing(k): its own ring, released right after this read
-        mbar_wait(&ws_ffull()[q % WS_FS], (uint32_t)(q / WS_FS) & 1u);
+        if (!FAST) ws_cwait(&ws_ffull()[q % WS_FS], (uint32_t)(q / WS_FS) & 1u);
         const double *fs = ws_f() + (size_t)(q % WS_FS) * F_SLOT;
 #pragma unroll
         // own forcing: (ty, tx+1) of the FX-wide tile = aux-tile index - AXW
@@ -218,8 +282,10 @@ __device__ __forceinline__ void ws_step(SegW &g, const Params &P, int k, int q, 
     // and plane k+2's tile has landed (own column read at the end of the
     // step); plane k+2's aux is not needed yet, so its evaluation overlaps
     // this step
-    mbar_wait(&ws_afull()[(q + 1) % WS_US], (uint32_t)((q + 1) / WS_US) & 1u);
-    mbar_wait(&ws_full()[(q + 2) % WS_US], (uint32_t)((q + 2) / WS_US) & 1u);
+    if (!FAST) {
+        ws_cwait(&ws_afull()[(q + 1) % WS_US], (uint32_t)((q + 1) / WS_US) & 1u);
+        ws_cwait(&ws_full()[(q + 2) % WS_US], (uint32_t)((q + 2) / WS_US) & 1u);
+    }
     const double *const s2 = su + (size_t)((q + 2) % WS_US) * U_SLOT;
     double an[5];
     const double (&wz)[5] = g.a[Z];
@@ -243,7 +309,7 @@ __device__ __forceinline__ void ws_step(SegW &g, const Params &P, int k, int q, 
             p.u[m] = g.a[PI][m];
             qn.u[m] = g.a[Q][m];
         }
-        if (PEER && k + 1 >= P.pk_hi) {  // f2: plane k+1 is the upper neighbour's
+        if (PEER && !FAST && k + 1 >= P.pk_hi) {  // f2: plane k+1 is the upper neighbour's
             aux_of(p.u[0], p.u[1], p.u[2], p.u[3], p.rho, p.sq);
         } else {
             const double2 o1 = ax[(size_t)((q + 1) % WS_US) * A_SLOT + g.ac];  // plane k+1
@@ -265,10 +331,21 @@ __device__ __forceinline__ void ws_step(SegW &g, const Params &P, int k, int q, 
         double t[5];
         {
             double pp[5], qq[5];
-            if (g.mid_x) {
+            if (FAST) {  // the table form for every tile (mid tiles: offsets 2, weights -4/6/-4)
+                const int xo = g.xo;
+                load5(pp, s, g.uc + (xo & 0xff));
+                load5(qq, s, g.uc - ((xo >> 8) & 0xff));
+                diss_terms_table(t, qq, qn.u, wz, p.u, pp, (xo & (1 << 16)) ? -4.0 : 0.0,
+                                 (xo & (1 << 17)) ? 5.0 : 6.0, (xo & (1 << 18)) ? -4.0 : 0.0);
+            } else if (g.mid_x) {
+#if SAFARA_WS_PROBE == 2  // timing probe: no xi dissipation loads / terms (wrong rhs)
+#pragma unroll
+                for (int m = 0; m < 5; ++m) t[m] = 0.0;
+#else
                 load5(pp, s, g.uc + 2);
                 load5(qq, s, g.uc - 2);
                 diss_terms<false>(t, qq, qn.u, wz, p.u, pp, Cases{});
+#endif
             } else {
 #if SAFARA_WS_XOREG
                 const int xo = g.xo;
@@ -282,7 +359,9 @@ __device__ __forceinline__ void ws_step(SegW &g, const Params &P, int k, int q, 
             }
         }
         flux_dir<1, false, UD>(acc, wz, vc, qsc, pc, p, qn, C, 0);
+#if SAFARA_WS_PROBE != 2
         diss_apply(acc, t, C.dssp);
+#endif
     }
     {   // eta
         Nb p, qn;
@@ -296,7 +375,10 @@ __device__ __forceinline__ void ws_step(SegW &g, const Params &P, int k, int q, 
             double pp[5], qq[5];
             load5(pp, s, g.uc + 2 * UX);
             load5(qq, s, g.uc - 2 * UX);
-            diss_terms_case(t, qq, qn.u, wz, p.u, pp, g.ycase);
+            if (FAST)
+                diss_eta_coef(t, qq, qn.u, wz, p.u, pp, c_eta_coef[g.ycase]);
+            else
+                diss_terms_case(t, qq, qn.u, wz, p.u, pp, g.ycase);
         }
         // every read of plane k's slot (u, forcing, aux) is done: release it
         __syncwarp();
@@ -307,13 +389,14 @@ __device__ __forceinline__ void ws_step(SegW &g, const Params &P, int k, int q, 
 #if !SAFARA_ZETA_FIRST
     zeta();
 #endif
-    if (PEER && k + 2 >= P.pk_hi)
+    if (PEER && !FAST && k + 2 >= P.pk_hi)
         peer_col(an, P, k + 2, g.colo);  // f2: the upper neighbour's own column
     else
         load5(an, s2, g.uc);
+#if SAFARA_WS_PROBE != 1  // 1: timing probe without the zeta dissipation (wrong rhs)
     {
         double t_z[5];
-        if (is_mid(k, P.nz)) {
+        if (FAST || is_mid(k, P.nz)) {
 #pragma unroll
             for (int m = 0; m < 5; ++m) t_z[m] = __fma_rn(-4.0, g.a[PI][m], g.tp[m]) + an[m];
         } else {
@@ -327,18 +410,37 @@ __device__ __forceinline__ void ws_step(SegW &g, const Params &P, int k, int q, 
         }
         diss_apply(acc, t_z, C.dssp);
     }
-    if (g.active) {
+#endif
+    if (FAST) {  // predicated stores: no branch
         double *rp = g.rptr;
 #pragma unroll
         for (int m = 0; m < 5; ++m) {
             const double v = acc[m] * C.dt;
+            st_cs_pred(rp, v, g.active);
+            if (NORM) {
+                const double va = g.active ? v : 0.0;
+                g.ss[m] = __fma_rn(va, va, g.ss[m]);
+            }
+            rp += SM(r);
+        }
+    } else if (g.active) {
+        double *rp = g.rptr;
+#pragma unroll
+        for (int m = 0; m < 5; ++m) {
+            const double v = acc[m] * C.dt;
+#if SAFARA_WS_STORE == 0
             __stcs(rp, v);
+#else
+            *rp = v;
+#endif
             if (NORM) g.ss[m] = __fma_rn(v, v, g.ss[m]);  // f1: NPB rhs_norm numerator
             rp += SM(r);
         }
     }
     g.rptr += SK(r);
-    zeta_partial(g.tp, g.a[Q], g.a[Z], g.a[PI], k + 1, P.nz, is_mid(k + 1, P.nz));
+#if SAFARA_WS_PROBE != 1
+    zeta_partial(g.tp, g.a[Q], g.a[Z], g.a[PI], k + 1, P.nz, FAST || is_mid(k + 1, P.nz));
+#endif
 #pragma unroll
     for (int m = 0; m < 5; ++m) g.a[Q][m] = an[m];
     g.rq = r0;  // plane k is plane k-1 of the next step
@@ -454,12 +556,25 @@ __device__ __forceinline__ void ws_consumer(const Params &P) {
 #pragma unroll
     for (int m = 0; m < 5; ++m) g.ss[m] = 0.0;
     int k = ka, q = 0;
+#if SAFARA_WS_FAST
+    // planes whose step can run FAST: k and k+1 interior in zeta and plane
+    // k+2 local (f2); CTA-uniform, so one uniform branch per step
+    const int kf_lo = 3, kf_hi = min(P.nz - 5, PEER ? P.pk_hi - 3 : P.nz);
+#define WS_STEP(RR, KK, QQ)                                                  \
+    if ((KK) >= kf_lo && (KK) <= kf_hi)                                      \
+        ws_step<RR, UD, AUX, NORM, PEER, true>(g, P, KK, QQ, ka);           \
+    else                                                                     \
+        ws_step<RR, UD, AUX, NORM, PEER, false>(g, P, KK, QQ, ka);
+#else
+#define WS_STEP(RR, KK, QQ) ws_step<RR, UD, AUX, NORM, PEER, false>(g, P, KK, QQ, ka);
+#endif
 #pragma unroll 1
     for (; k + 3 <= kb; k += 3, q += 3) {
-        ws_step<0, UD, AUX, NORM, PEER>(g, P, k, q, ka);
-        ws_step<1, UD, AUX, NORM, PEER>(g, P, k + 1, q + 1, ka);
-        ws_step<2, UD, AUX, NORM, PEER>(g, P, k + 2, q + 2, ka);
+        WS_STEP(0, k, q)
+        WS_STEP(1, k + 1, q + 1)
+        WS_STEP(2, k + 2, q + 2)
     }
+#undef WS_STEP
     if (k < kb) {
         ws_step<0, UD, AUX, NORM, PEER>(g, P, k, q, ka);
         if (k + 1 < kb) ws_step<1, UD, AUX, NORM, PEER>(g, P, k + 1, q + 1, ka);

@@ -60,3 +60,26 @@ def test_seismic_errors():
     big = sr.Dims3(nx, ny, nz, 8, 1 << 30)
     assert L.safara_seismic_dz(*p, ctypes.byref(big), 1.0, None) == -5          # `small`
     assert L.safara_seismic_dz(*p, ctypes.byref(d), 1.0, None) == 0
+
+
+@pytest.mark.parametrize("h", [0.37, 0.01, 1.0 / 3.0, 3.0, 1e-7, 12345.678, 2.0 ** -20, 0.7071067811865476])
+def test_seismic_bitwise_wide_range(h):
+    """Differences spanning +-250 binades and several spacings h: the division
+    (IEEE x/h, or the library's correction form from RN(1/h)) must stay
+    bit-identical to the oracle's IEEE division for every value."""
+    nx, ny, nz = 67, 33, 41
+    r = np.random.default_rng(int(h * 1e6) % 2**31)
+    v = [r.standard_normal((nz, ny, nx)) * np.exp2(r.integers(-250, 250, (nz, ny, nx)))
+         for _ in range(3)]
+    sy = sr.pitch(nx)
+    dv = []
+    for a in v:
+        t = torch.zeros((nz, ny, sy), dtype=torch.float64)
+        t[..., :nx] = torch.from_numpy(a)
+        dv.append(t.cuda())
+    out = torch.full((nz, ny, sy), float("nan"), dtype=torch.float64, device="cuda")
+    sr.seismic_dz(*dv, out, h, nx)
+    g = out[..., :nx].cpu().numpy()
+    o = oracle.seismic_dz(*v, h)
+    assert np.array_equal(np.isnan(g), np.isnan(o))
+    assert np.array_equal(np.nan_to_num(g), np.nan_to_num(o))
