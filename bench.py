@@ -183,6 +183,44 @@ class ClockSampler:
                 "reasons": sorted(reasons)}
 
 
+class NvmlEnergy:
+    """NVML total-energy counter (mJ) of one GPU; None when NVML is absent."""
+
+    def __init__(self, gpu_index):
+        self.h = None
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(gpu_index)
+        except Exception:
+            self.h = None
+
+    def mj(self):
+        if self.h is None:
+            return None
+        try:
+            return self.nv.nvmlDeviceGetTotalEnergyConsumption(self.h)
+        except Exception:
+            return None
+
+
+def power_summary(e0, e1, secs, passes, clocks, frac):
+    """Board energy per pass over the untimed soak that precedes the timed
+    region (same workload, back to back): the 1 kW cap binds, so joules per
+    pass -- not cycles -- set the pass time.  `frac_at_sm_max`
+    is a labelled what-if: the roofline fraction scaled by sm_max / sm_mhz,
+    i.e. the same cycles at the unthrottled clock; it is not a measurement."""
+    out = {"soak_s": round(secs, 3), "soak_passes": passes}
+    if e0 is not None and e1 is not None and passes > 0 and secs > 0:
+        out["w_mean"] = round((e1 - e0) / secs / 1e3, 1)
+        out["mj_per_pass"] = round((e1 - e0) / passes, 3)
+    sm, smx = clocks.get("sm_mhz"), clocks.get("sm_max_mhz")
+    if sm and smx:
+        out["frac_at_sm_max"] = round(frac * smx / sm, 4)
+    return out
+
+
 def cpu_oracle_time(inp, max_seconds=12.0, threads=None, min_passes=1):
     """Time the oracle as it stands on the host cores (full passes)."""
     import oracle
@@ -375,11 +413,15 @@ def run_single(args):
 
     sampler = ClockSampler(0)
     sampler.start()
+    nvml = NvmlEnergy(0)
+    e_soak0, t_soak0, n_soak = nvml.mj(), time.time(), 0
     t_end = time.time() + args.soak_s
     while time.time() < t_end:
         for _ in range(50):
             step()
+        n_soak += 50 * (G if graph is not None else 1)
         torch.cuda.synchronize()
+    e_soak1, t_soak1 = nvml.mj(), time.time()
 
     # timed region: K steps, per-launch events on the launching stream
     ev = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps + 1)]
@@ -454,6 +496,8 @@ def run_single(args):
                           "note": "algorithmic flops (430/pt); the FP64 pipe is the "
                                   "near-binding second roofline (DESIGN.md §5)"},
         "clocks": clocks,
+        "power": power_summary(e_soak0, e_soak1, t_soak1 - t_soak0, n_soak, clocks,
+                               achieved / peak),
         "e2e": {"value": pts / (e2e_ms * 1e-3) / 1e9, "unit": "Gpt/s",
                 "h2d_bytes_per_step": 2 * nbytes, "d2h_bytes_per_step": nbytes,
                 "ms_per_step": e2e_ms},

@@ -48,6 +48,9 @@ __device__ __forceinline__ void ws_pwait(uint64_t *bar, uint32_t parity) {
 #ifndef SAFARA_WS_PROBE
 #define SAFARA_WS_PROBE 0  // timing probes (wrong rhs): 1 no zeta dissipation, 2 no xi dissipation (mid tiles)
 #endif
+#ifndef SAFARA_WS_NORM_PROBE
+#define SAFARA_WS_NORM_PROBE 0  // timing probe: the fused norm without its in-loop accumulation (wrong norm)
+#endif
 #ifndef SAFARA_WS_CSLEEP
 #define SAFARA_WS_CSLEEP 0      // consumer waits: suspend-time hint (ns), 0 = plain try_wait spin
 #endif
@@ -433,7 +436,7 @@ __device__ __forceinline__ void ws_step(SegW &g, const Params &P, int k, int q, 
 #else
             *rp = v;
 #endif
-            if (NORM) g.ss[m] = __fma_rn(v, v, g.ss[m]);  // f1: NPB rhs_norm numerator
+            if (NORM && !SAFARA_WS_NORM_PROBE) g.ss[m] = __fma_rn(v, v, g.ss[m]);  // f1: NPB rhs_norm numerator
             rp += SM(r);
         }
     }
@@ -457,6 +460,8 @@ __device__ __forceinline__ void ws_step(SegW &g, const Params &P, int k, int q, 
 // launch), leaving the counter at 0.
 __shared__ double ws_red[TY][5];
 __shared__ int ws_last;
+constexpr int WS_NRED = 25;  // last-CTA reduction: threads per component
+__shared__ double ws_red2[5][WS_NRED];
 constexpr int WS_NORM_BAR = 2;
 
 __device__ __forceinline__ void ws_norm_consumer(const double (&ss)[5], int tid) {
@@ -481,18 +486,38 @@ __device__ __forceinline__ void ws_norm_producer(const Params &P) {
     }
     asm volatile("bar.sync 3, 128;" ::: "memory");  // producers: partials stored
     if (pt == 0) {
-        __threadfence();
-        const unsigned long long old = atomicAdd(P.norm_ctr, 1ull);
+        // one acq_rel atomic instead of fence + atomic: releases this CTA's
+        // partials (ordered before it by the barrier; release is cumulative)
+        // and, for the last CTA, acquires every other CTA's
+        unsigned long long old;
+        asm volatile("atom.acq_rel.gpu.global.add.u64 %0, [%1], 1;"
+                     : "=l"(old) : "l"(P.norm_ctr) : "memory");
         ws_last = old == (unsigned long long)P.ncta - 1;
     }
     asm volatile("bar.sync 3, 128;" ::: "memory");
-    if (ws_last && pt < 5) {
-        __threadfence();
-        double t = 0.0;
-        for (int b = 0; b < P.ncta; ++b) t += __ldcg(P.norm_part + pt * P.ncta + b);
-        P.norm_out[pt] = P.norm_npts > 0.0 ? sqrt(t / P.norm_npts) : t;
+    if (ws_last) {
+        // the last CTA: 125 threads sum the CTA partials of component
+        // pt / 25 strided by 25 (fixed order, loads independent), then 5
+        // threads add the 25 sums in order -- deterministic for a given grid,
+        // and ~2 dependent L2 round trips instead of ncta (the partials
+        // were acquired by thread 0's atomic; the barrier orders the loads)
+        if (pt < 5 * WS_NRED) {
+            const int m = pt / WS_NRED, s0 = pt - m * WS_NRED;
+            const double *part = P.norm_part + m * P.ncta;
+            double t = 0.0;
+#pragma unroll 8
+            for (int b = s0; b < P.ncta; b += WS_NRED) t += __ldcg(part + b);
+            ws_red2[m][s0] = t;
+        }
+        asm volatile("bar.sync 3, 128;" ::: "memory");
+        if (pt < 5) {
+            double t = 0.0;
+#pragma unroll
+            for (int s = 0; s < WS_NRED; ++s) t += ws_red2[pt][s];
+            P.norm_out[pt] = P.norm_npts > 0.0 ? sqrt(t / P.norm_npts) : t;
+        }
+        if (pt == 0) *P.norm_ctr = 0ull;
     }
-    if (ws_last && pt == 0) *P.norm_ctr = 0ull;
 }
 
 template <bool UD, bool AUX, bool NORM, bool PEER>
