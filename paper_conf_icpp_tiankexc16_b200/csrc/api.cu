@@ -61,6 +61,7 @@ struct Tune {
     int peer_bias_maxpart = 6;  // peer_bias only for k-parts of at most this many planes
     int peer_timeout_ms = 30000;  // f2 flag waits: give up and trap after this long
     int ws = 1;  // warp-specialised kernel (rhs_ws.cuh) where it applies (0: round-1 kernel)
+    int iface = 1;  // WS launches: edge column tiles write the i-face columns (SAFARA_IFACE)
 } g_tune;
 
 int env_int(const char *name, int dflt) {
@@ -351,6 +352,7 @@ int launch(const double *u, const double *f, double *r, const safara_dims_t &d, 
     // without the f1 aux output or the f2 peer halo
     const bool ws = g_tune.ws && lockstep && p.parts > 0 && p.n0 == p.nplanes &&
                     !(peer && aux);
+    p.iface_tiles = ws && !aux && g_tune.iface ? 1 : 0;
 
     // f1 fused rhs_norm: the warp-specialised kernel with NAS coefficients
     // writes per-CTA partial sums; otherwise the caller runs the two-pass norm
@@ -463,6 +465,7 @@ int safara_rhs_init(int device) {
     g_tune.peer_bias_maxpart = env_int("SAFARA_PEER_BIAS_MAXPART", g_tune.peer_bias_maxpart);
     g_tune.peer_timeout_ms = std::max(1, env_int("SAFARA_PEER_TIMEOUT_MS", g_tune.peer_timeout_ms));
     g_tune.ws = env_int("SAFARA_WS", g_tune.ws);
+    g_tune.iface = env_int("SAFARA_IFACE", g_tune.iface);
     int major = 0, minor = 0, sms = 0;
     if (cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, device) ||
         cudaDeviceGetAttribute(&minor, cudaDevAttrComputeCapabilityMinor, device) ||

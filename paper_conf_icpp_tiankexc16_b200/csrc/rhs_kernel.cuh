@@ -624,6 +624,8 @@ __device__ __forceinline__ void copy_faces(const Params &P, int cta, int nctas) 
                         e -= 2 * nx;
                         if (e < ny - 2) { i = 0; j = 1 + e; }
                         else { i = nx - 1; j = 1 + e - (ny - 2); }
+                        // written by the edge column tiles of this launch
+                        if (P.iface_tiles && kl + P.k0 >= P.ka0 && kl + P.k0 < P.kb0) continue;
                     }
                 } else {
                     const int e = ti - (int)nper;

@@ -193,6 +193,8 @@ struct SegW {
     double *rptr;
     int uc, ac;
     bool active, mid_x;
+    int fidx;        // i-face copy (P.iface_tiles): forcing-tile index of this lane's value, or -1
+    double *fptr;    //   and its rhs address at the current plane
     int ycase;
 #if SAFARA_WS_XOREG
     int xo;
@@ -278,6 +280,10 @@ __device__ __forceinline__ void ws_step(SegW &g, const Params &P, int k, int q, 
         // own forcing: (ty, tx+1) of the FX-wide tile = aux-tile index - AXW
         static_assert(FX == AXW, "forcing and aux tiles share the row width");
         for (int m = 0; m < 5; ++m) acc[m] = fs[m * TY * FX - AXW + g.ac];
+        if (g.fidx >= 0) {  // one i-face value of this row: rhs = forcing (reading c3)
+            __stcs(g.fptr, fs[g.fidx]);
+            g.fptr += SK(r);
+        }
         __syncwarp();
         if ((threadIdx.x & 31) == 0) mbar_arrive(&ws_fempty()[q % WS_FS]);
     }
@@ -538,6 +544,23 @@ __device__ __forceinline__ void ws_consumer(const Params &P) {
     const int nx_s = reread(P.nx), ny_s = reread(P.ny);
     SegW g;
     g.active = (i <= nx_s - 2) && (j <= ny_s - 2);
+    // the i-face columns (P.iface_tiles): in the first column tile lanes 0..4
+    // copy component `lane` of rhs(0, j, k) = forcing(0, j, k), in the last
+    // column tile lanes 5..9 that of i = nx-1 (rows 1..ny-2); the forcing
+    // tile's columns i0-1 .. i0+TX hold both, so each warp adds one shared
+    // load and one store per step (5 lanes active)
+    g.fidx = -1;
+    g.fptr = nullptr;
+    if (!AUX && P.iface_tiles && j <= ny_s - 2) {
+        const int ctile = (col % P.ntx);
+        int fi = -1, m = -1;
+        if (tx < 5 && ctile == 0) { fi = 0; m = tx; }
+        else if (tx >= 5 && tx < 10 && ctile == P.ntx - 1) { fi = nx_s - 1; m = tx - 5; }
+        if (fi >= 0) {
+            g.fidx = m * TY * FX + ty * FX + (fi - (i0 - 1));
+            g.fptr = P.r + ((idx_t)fi + SY(r) * j + SM(r) * m + SK(r) * (ka - P.k0));
+        }
+    }
     g.uc = (ty + 2) * UX + (tx + HX);
     g.ac = (ty + 1) * AXW + (tx + 1);
     g.mid_x = is_mid(i0, P.nx) && is_mid(i0 + TX - 1, P.nx);

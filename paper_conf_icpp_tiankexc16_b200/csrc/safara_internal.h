@@ -109,6 +109,10 @@ struct Params {
     int split_bias;        // lockstep: planes the last k-part gives to the others (f2)
     int units;             // ncol*nplanes (column-plane work items, < 2^31)
     int fk_lo, fk_hi;      // local planes whose boundary faces this launch copies
+    int iface_tiles;       // 1: the i-face columns of the marched planes [ka0, kb0), rows
+                           // 1..ny-2, are written by the edge column tiles (warp-specialised
+                           // kernel, from the forcing tile in shared memory); the face
+                           // CTAs skip them
     int pos_j, pos_m, pos_k;  // tensor-map dimension holding j, m, k
     const double *u;       // u buffer base (local plane 0)
     const double *f;       // forcing base (local plane 0)
