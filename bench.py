@@ -63,6 +63,9 @@ def parse():
                          "(back-to-back graph replays raise the power draw and the cap takes "
                          "it back in clock), 20 for the fused-halo multi-GPU path (per-rank "
                          "passes of 10-20 us, where the launch gap is 10%%)")
+    ap.add_argument("--e2e-canonical", action="store_true",
+                    help="e2e through safara_rhs_host on the canonical pitched layout "
+                         "(default: the unpadded sy = nx layout via safara_rhs_host_ex when nx is even)")
     ap.add_argument("--slab-sim", type=int, default=0, metavar="P",
                     help="one GPU: time the middle rank's fused-halo pass of a P-way "
                          "z-split (neighbour slabs resident on the same GPU) next to the "
@@ -456,18 +459,40 @@ def run_single(args):
 
     # e2e: host (pinned) buffers through the C ABI, H2D + pass + D2H per step
     e2e_ms, nbytes = float("nan"), 0
+    e2e_layout = None
     if args.e2e_steps > 0 and args.workload == "rhs":
-        hu, hf = sr.pack(inp.u, pin=True), sr.pack(inp.forcing, pin=True)
-        hr = torch.empty(hu.shape, dtype=torch.float64).pin_memory()
+        import numpy as np
+        if nx % 2 == 0 and not args.e2e_canonical:
+            # the NAS-native unpadded layout (sy = nx) through safara_rhs_host_ex:
+            # 3.6 % fewer PCIe bytes than the canonical pitch at class C
+            def host(a):
+                t = torch.empty((nz, 5, ny, nx), dtype=torch.float64).pin_memory()
+                t.copy_(torch.from_numpy(np.ascontiguousarray(a)).permute(0, 3, 1, 2))
+                return t
+            hu, hf = host(inp.u), host(inp.forcing)
+            hr = torch.empty(hu.shape, dtype=torch.float64).pin_memory()
+            eu, ef, er = (torch.empty(hu.shape, dtype=torch.float64, device="cuda") for _ in range(3))
+            dd = sr.Dims(nx, ny, nz, nx, ny * nx, 5 * ny * nx)
+            e2e_layout = "unpadded sy = nx (safara_rhs_host_ex)"
+
+            def e2e_step():
+                sr.rhs_host_ex(hu, hf, hr, eu, ef, er, dd, c, strict=args.strict,
+                               nchunks=args.e2e_chunks, stream=stream)
+        else:
+            hu, hf = sr.pack(inp.u, pin=True), sr.pack(inp.forcing, pin=True)
+            hr = torch.empty(hu.shape, dtype=torch.float64).pin_memory()
+            e2e_layout = f"canonical pitch sy = {sr.pitch(nx)} (safara_rhs_host)"
+
+            def e2e_step():
+                sr.rhs_host(hu, hf, hr, du, df, dr, nx, c, strict=args.strict,
+                            nchunks=args.e2e_chunks, stream=stream)
         for _ in range(2):
-            sr.rhs_host(hu, hf, hr, du, df, dr, nx, c, strict=args.strict,
-                        nchunks=args.e2e_chunks, stream=stream)
+            e2e_step()
         torch.cuda.synchronize()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)
         for _ in range(args.e2e_steps):
-            sr.rhs_host(hu, hf, hr, du, df, dr, nx, c, strict=args.strict,
-                        nchunks=args.e2e_chunks, stream=stream)
+            e2e_step()
         e1.record(stream)
         torch.cuda.synchronize()
         e2e_ms = e0.elapsed_time(e1) / args.e2e_steps
@@ -500,7 +525,7 @@ def run_single(args):
                                achieved / peak),
         "e2e": {"value": pts / (e2e_ms * 1e-3) / 1e9, "unit": "Gpt/s",
                 "h2d_bytes_per_step": 2 * nbytes, "d2h_bytes_per_step": nbytes,
-                "ms_per_step": e2e_ms},
+                "ms_per_step": e2e_ms, "host_layout": e2e_layout},
         "gpu_launches": launches,
         "kernel": sr.kernel_info(args.strict),
     }

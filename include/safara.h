@@ -449,6 +449,18 @@ int safara_rhs_host(const double *u_host, const double *forcing_host,
                     const safara_coeffs_t *coeffs, int flags, int nchunks,
                     void *stream);
 
+/* The same with an explicit shared descriptor (`dim` clause) for the host and
+ * device arrays, e.g. the unpadded NAS-native layout sy = nx (nx even) that
+ * moves 3.6 % fewer PCIe bytes at class C than the canonical pitch.  k must
+ * be the outermost dimension (sk >= 5*sm: the k-chunks are contiguous byte
+ * ranges); otherwise as safara_rhs_host (validation as safara_rhs_ex, plus
+ * SAFARA_ERR_LAYOUT when k is not outermost).                               */
+int safara_rhs_host_ex(const double *u_host, const double *forcing_host,
+                       double *rhs_host, double *u_dev, double *forcing_dev,
+                       double *rhs_dev, const safara_dims_t *dims,
+                       const safara_coeffs_t *coeffs, int flags, int nchunks,
+                       void *stream);
+
 /* Number of kernel launches issued by this process since load.            */
 int64_t safara_launch_count(void);
 

@@ -89,6 +89,8 @@ _SIGS = {
                          ctypes.POINTER(Coeffs), ctypes.c_int, ctypes.c_int, _dp], ctypes.c_int),
     "safara_rhs_host": ([_dp] * 6 + [ctypes.c_int] * 3 + [ctypes.POINTER(Coeffs), ctypes.c_int,
                                                            ctypes.c_int, _dp], ctypes.c_int),
+    "safara_rhs_host_ex": ([_dp] * 6 + [ctypes.POINTER(Dims), ctypes.POINTER(Coeffs), ctypes.c_int,
+                            ctypes.c_int, _dp], ctypes.c_int),
     "safara_rhs_aux": ([_dp, _dp, _dp, _dp, ctypes.c_int, ctypes.POINTER(Dims),
                         ctypes.POINTER(Coeffs), ctypes.c_int, _dp], ctypes.c_int),
     "safara_rhs_slab_aux": ([_dp, _dp, _dp, _dp, ctypes.c_int, ctypes.POINTER(Dims), ctypes.c_int,

@@ -731,12 +731,23 @@ int safara_rhs_slab_aux(const double *u_slab, const double *forcing_slab, double
 int safara_rhs_host(const double *u_host, const double *forcing_host, double *rhs_host,
                     double *u_dev, double *forcing_dev, double *rhs_dev, int nx, int ny, int nz,
                     const safara_coeffs_t *coeffs, int flags, int nchunks, void *stream) {
-    if (!u_host || !forcing_host || !rhs_host) return SAFARA_ERR_ARG;
     safara_dims_t d;
     int rc = safara_dims_canonical(nx, ny, nz, &d);
     if (rc) return rc;
-    rc = validate(&d, nz);
+    return safara_rhs_host_ex(u_host, forcing_host, rhs_host, u_dev, forcing_dev, rhs_dev, &d,
+                              coeffs, flags, nchunks, stream);
+}
+
+int safara_rhs_host_ex(const double *u_host, const double *forcing_host, double *rhs_host,
+                       double *u_dev, double *forcing_dev, double *rhs_dev,
+                       const safara_dims_t *dims, const safara_coeffs_t *coeffs, int flags,
+                       int nchunks, void *stream) {
+    if (!u_host || !forcing_host || !rhs_host || !dims) return SAFARA_ERR_ARG;
+    const safara_dims_t d = *dims;
+    const int nz = d.nz;
+    int rc = validate(&d, nz);
     if (rc) return rc;
+    if ((long long)d.sk < 5LL * d.sm) return SAFARA_ERR_LAYOUT;  // k outermost: chunks are byte ranges
     const long long bytes = (long long)d.sk * nz * (long long)sizeof(double);
     rc = check_ptrs(u_dev, bytes, forcing_dev, bytes, rhs_dev, bytes);
     if (rc) return rc;

@@ -289,6 +289,29 @@ def rhs_host(u_host: torch.Tensor, f_host: torch.Tensor, r_host: torch.Tensor,
     return r_host
 
 
+def rhs_host_ex(u_host: torch.Tensor, f_host: torch.Tensor, r_host: torch.Tensor,
+                u_dev: torch.Tensor, f_dev: torch.Tensor, r_dev: torch.Tensor, dims: Dims,
+                coeffs: Coeffs, strict: bool = False, nchunks: int = 8, stream=None):
+    """End-to-end pass on host (pinned) arrays in the layout `dims` describes
+    (e.g. the unpadded sy = nx layout) through device buffers of the same layout."""
+    need = (_max_offset(dims, dims.nz) + 1)
+    for t, n in ((u_host, "u_host"), (f_host, "f_host"), (r_host, "r_host")):
+        if t.dtype != torch.float64 or not t.is_contiguous() or t.device.type != "cpu":
+            raise ValueError(f"{n}: contiguous float64 CPU tensor expected")
+        if t.numel() < need:
+            raise ValueError(f"{n}: {t.numel()} elements < the descriptor's {need}")
+    for t, n in ((u_dev, "u_dev"), (f_dev, "f_dev"), (r_dev, "r_dev")):
+        _check_field(t, n)
+        if t.numel() < need:
+            raise ValueError(f"{n}: {t.numel()} elements < the descriptor's {need}")
+    flags = SAFARA_FLAG_STRICT if strict else 0
+    check(lib().safara_rhs_host_ex(u_host.data_ptr(), f_host.data_ptr(), r_host.data_ptr(),
+                                   u_dev.data_ptr(), f_dev.data_ptr(), r_dev.data_ptr(),
+                                   ctypes.byref(dims), ctypes.byref(coeffs), flags, int(nchunks),
+                                   _stream_ptr(stream)), "safara_rhs_host_ex")
+    return r_host
+
+
 def launch_count() -> int:
     return int(lib().safara_launch_count())
 

@@ -316,3 +316,28 @@ def test_warp_specialised_kernel_parity():
                        env=dict(os.environ, SAFARA_WS="1"), capture_output=True, text=True,
                        timeout=600)
     assert r.returncode == 0 and "ws ok" in r.stdout, r.stderr[-2000:]
+
+
+@pytest.mark.parametrize("cls,nchunks", [(("SP", "W"), 3), (("BT", "C"), 8)])
+def test_host_e2e_unpadded_descriptor(cls, nchunks):
+    """safara_rhs_host_ex on the unpadded NAS-native layout (sy = nx, the
+    `dim` descriptor given explicitly): STRICT bit-identical to the oracle
+    through host buffers, k-chunked copies and the kernel on sy = nx rows."""
+    inp = nasgen.make_class(*cls, seed=8)
+    nz, ny, nx, _ = inp.u.shape
+    assert nx % 2 == 0
+
+    def host(a):
+        t = torch.empty((nz, 5, ny, nx), dtype=torch.float64).pin_memory()
+        t.copy_(torch.from_numpy(np.ascontiguousarray(a)).permute(0, 3, 1, 2))
+        return t
+
+    hu, hf = host(inp.u), host(inp.forcing)
+    hr = torch.zeros_like(hu).pin_memory()
+    du, df, dr = (torch.empty(hu.shape, dtype=torch.float64, device="cuda") for _ in range(3))
+    d = sr.Dims(nx, ny, nz, nx, ny * nx, 5 * ny * nx)
+    c = sr.coeffs_nas(nx, ny, nz, inp.dt)
+    sr.rhs_host_ex(hu, hf, hr, du, df, dr, d, c, strict=True, nchunks=nchunks)
+    torch.cuda.synchronize()
+    got = hr.permute(0, 2, 3, 1).numpy()
+    assert np.array_equal(got, oracle_rhs(inp))
