@@ -63,6 +63,9 @@ def parse():
                          "(back-to-back graph replays raise the power draw and the cap takes "
                          "it back in clock), 20 for the fused-halo multi-GPU path (per-rank "
                          "passes of 10-20 us, where the launch gap is 10%%)")
+    ap.add_argument("--e2e-serial", action="store_true",
+                    help="e2e steps without SAFARA_FLAG_PIPELINE (each step's H2D waits for "
+                         "the previous step's D2H tail)")
     ap.add_argument("--e2e-canonical", action="store_true",
                     help="e2e through safara_rhs_host on the canonical pitched layout "
                          "(default: the unpadded sy = nx layout via safara_rhs_host_ex when nx is even)")
@@ -477,7 +480,8 @@ def run_single(args):
 
             def e2e_step():
                 sr.rhs_host_ex(hu, hf, hr, eu, ef, er, dd, c, strict=args.strict,
-                               nchunks=args.e2e_chunks, stream=stream)
+                               nchunks=args.e2e_chunks, stream=stream,
+                               pipeline=not args.e2e_serial)
         else:
             hu, hf = sr.pack(inp.u, pin=True), sr.pack(inp.forcing, pin=True)
             hr = torch.empty(hu.shape, dtype=torch.float64).pin_memory()
@@ -485,7 +489,8 @@ def run_single(args):
 
             def e2e_step():
                 sr.rhs_host(hu, hf, hr, du, df, dr, nx, c, strict=args.strict,
-                            nchunks=args.e2e_chunks, stream=stream)
+                            nchunks=args.e2e_chunks, stream=stream,
+                            pipeline=not args.e2e_serial)
         for _ in range(2):
             e2e_step()
         torch.cuda.synchronize()
@@ -525,7 +530,8 @@ def run_single(args):
                                achieved / peak),
         "e2e": {"value": pts / (e2e_ms * 1e-3) / 1e9, "unit": "Gpt/s",
                 "h2d_bytes_per_step": 2 * nbytes, "d2h_bytes_per_step": nbytes,
-                "ms_per_step": e2e_ms, "host_layout": e2e_layout},
+                "ms_per_step": e2e_ms, "host_layout": e2e_layout,
+                "pipelined": bool(args.e2e_steps > 0 and not args.e2e_serial)},
         "gpu_launches": launches,
         "kernel": sr.kernel_info(args.strict),
     }

@@ -60,6 +60,15 @@ enum {
 #define SAFARA_FLAG_STRICT 0x1  /* bit-identical to the NAS evaluation order:
                                    no FMA contraction except where the product
                                    is an exact power-of-two scaling           */
+#define SAFARA_FLAG_PIPELINE 0x2 /* safara_rhs_host(_ex) only: consecutive
+                                   calls with this flag and the same device
+                                   buffers, chunking and stream form one
+                                   pipeline -- a call's H2D of chunk c starts
+                                   as soon as the previous call's kernels no
+                                   longer read those planes (not after the
+                                   previous call's D2H tail).  The caller must
+                                   not touch u_dev / forcing_dev between such
+                                   calls.                                     */
 
 /* The shared stride descriptor (`dim` + `small`).  Extents are the GLOBAL
  * grid; lower bounds are 0; sx == 1 implicitly.                              */
@@ -449,7 +458,11 @@ int safara_rhs_host(const double *u_host, const double *forcing_host,
                     const safara_coeffs_t *coeffs, int flags, int nchunks,
                     void *stream);
 
-/* The same with an explicit shared descriptor (`dim` clause) for the host and
+/* With SAFARA_FLAG_PIPELINE (see above) back-to-back calls keep the H2D copy
+ * engine busy across calls: the next call's first chunks are copied in while
+ * this call's last chunks are computed and copied out.
+ *
+ * The same with an explicit shared descriptor (`dim` clause) for the host and
  * device arrays, e.g. the unpadded NAS-native layout sy = nx (nx even) that
  * moves 3.6 % fewer PCIe bytes at class C than the canonical pitch.  k must
  * be the outermost dimension (sk >= 5*sm: the k-chunks are contiguous byte

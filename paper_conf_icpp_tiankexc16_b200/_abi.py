@@ -17,6 +17,7 @@ HEADER = os.path.join(os.path.dirname(PKG), "include", "safara.h")
 
 SAFARA_OK = 0
 SAFARA_FLAG_STRICT = 0x1
+SAFARA_FLAG_PIPELINE = 0x2
 SAFARA_PART_ALL, SAFARA_PART_INTERIOR, SAFARA_PART_EDGE = 0, 1, 2
 SAFARA_AUX_BT, SAFARA_AUX_SP = 6, 7
 

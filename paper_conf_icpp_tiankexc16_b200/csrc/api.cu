@@ -40,6 +40,14 @@ struct DeviceState {
     cudaStream_t h2d = nullptr, d2h = nullptr;
     cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
     cudaEvent_t ev_h[kMaxChunks] = {}, ev_c[kMaxChunks] = {};
+    // SAFARA_FLAG_PIPELINE: the previous pipelined host call (buffers, chunks,
+    // layout, stream); its ev_c events mark when its kernels stopped reading
+    struct {
+        bool valid = false;
+        const double *u = nullptr, *f = nullptr, *r = nullptr;
+        int C = 0, nz = 0, sk = 0;
+        void *stream = nullptr;
+    } pipe;
 };
 
 DeviceState g_dev[kMaxDevices];
@@ -743,6 +751,9 @@ int safara_rhs_host_ex(const double *u_host, const double *forcing_host, double 
                        const safara_dims_t *dims, const safara_coeffs_t *coeffs, int flags,
                        int nchunks, void *stream) {
     if (!u_host || !forcing_host || !rhs_host || !dims) return SAFARA_ERR_ARG;
+    if (flags & ~(SAFARA_FLAG_STRICT | SAFARA_FLAG_PIPELINE)) return SAFARA_ERR_ARG;
+    const bool pipeline = (flags & SAFARA_FLAG_PIPELINE) != 0;
+    flags &= SAFARA_FLAG_STRICT;
     const safara_dims_t d = *dims;
     const int nz = d.nz;
     int rc = validate(&d, nz);
@@ -763,12 +774,20 @@ int safara_rhs_host_ex(const double *u_host, const double *forcing_host, double 
     int C = std::max(1, std::min(std::min(nchunks, kMaxChunks), nz / 4));
     auto z = [&](int c) { return (int)((long long)nz * c / C); };
     const size_t plane = (size_t)d.sk * sizeof(double);
+    // pipelined continuation of the previous call: no fork on `stream` (whose
+    // tail is the previous call's D2H); each H2D chunk instead waits for the
+    // previous call's kernels that read its planes (chunks c-1 .. c+1)
+    const bool cont = pipeline && st.pipe.valid && st.pipe.u == u_dev &&
+                      st.pipe.f == forcing_dev && st.pipe.r == rhs_dev && st.pipe.C == C &&
+                      st.pipe.nz == nz && st.pipe.sk == d.sk && st.pipe.stream == stream;
+    st.pipe.valid = false;  // set again only when this call is fully enqueued
     bool ok = cudaEventRecord(st.ev_fork, s) == cudaSuccess &&
-              cudaStreamWaitEvent(st.h2d, st.ev_fork, 0) == cudaSuccess &&
-              cudaStreamWaitEvent(st.d2h, st.ev_fork, 0) == cudaSuccess;
+              cudaStreamWaitEvent(st.d2h, st.ev_fork, 0) == cudaSuccess &&
+              (cont || cudaStreamWaitEvent(st.h2d, st.ev_fork, 0) == cudaSuccess);
     for (int c = 0; ok && c < C; ++c) {
         const size_t off = (size_t)z(c) * d.sk, len = (size_t)(z(c + 1) - z(c)) * plane;
-        ok = cudaMemcpyAsync(u_dev + off, u_host + off, len, cudaMemcpyHostToDevice, st.h2d) ==
+        if (cont) ok = cudaStreamWaitEvent(st.h2d, st.ev_c[std::min(c + 1, C - 1)], 0) == cudaSuccess;
+        ok = ok && cudaMemcpyAsync(u_dev + off, u_host + off, len, cudaMemcpyHostToDevice, st.h2d) ==
                  cudaSuccess &&
              cudaMemcpyAsync(forcing_dev + off, forcing_host + off, len, cudaMemcpyHostToDevice,
                              st.h2d) == cudaSuccess &&
@@ -788,6 +807,9 @@ int safara_rhs_host_ex(const double *u_host, const double *forcing_host, double 
     }
     ok = ok && cudaEventRecord(st.ev_join, st.d2h) == cudaSuccess &&
          cudaStreamWaitEvent(s, st.ev_join, 0) == cudaSuccess;
+    st.pipe.valid = ok && pipeline;
+    st.pipe.u = u_dev; st.pipe.f = forcing_dev; st.pipe.r = rhs_dev;
+    st.pipe.C = C; st.pipe.nz = nz; st.pipe.sk = d.sk; st.pipe.stream = stream;
     return ok ? SAFARA_OK : SAFARA_ERR_CUDA;
 }
 

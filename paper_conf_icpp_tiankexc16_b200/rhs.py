@@ -13,7 +13,7 @@ import ctypes
 import numpy as np
 import torch
 
-from ._abi import (SAFARA_AUX_BT, SAFARA_AUX_SP, SAFARA_FLAG_STRICT, SAFARA_IPC_HANDLE_BYTES,
+from ._abi import (SAFARA_AUX_BT, SAFARA_AUX_SP, SAFARA_FLAG_STRICT, SAFARA_FLAG_PIPELINE, SAFARA_IPC_HANDLE_BYTES,
                    SAFARA_PART_ALL, SAFARA_UNIQUE_ID_BYTES, BtCoeffs, Coeffs, Dims, Dims3,
                    KernelInfo, Peer, check, lib)
 
@@ -275,13 +275,15 @@ def ipc_close(ptr: int, offset: int) -> None:
 
 def rhs_host(u_host: torch.Tensor, f_host: torch.Tensor, r_host: torch.Tensor,
              u_dev: torch.Tensor, f_dev: torch.Tensor, r_dev: torch.Tensor, nx: int,
-             coeffs: Coeffs, strict: bool = False, nchunks: int = 8, stream=None):
-    """End-to-end pass on host (pinned) canonical tensors through device buffers."""
+             coeffs: Coeffs, strict: bool = False, nchunks: int = 8, stream=None,
+             pipeline: bool = False):
+    """End-to-end pass on host (pinned) canonical tensors through device buffers
+    (pipeline: SAFARA_FLAG_PIPELINE, see include/safara.h)."""
     nz, ny = _canonical_fields(nx, ((u_host, "u_host"), (f_host, "f_host"), (r_host, "r_host")))
     for t, n in ((u_dev, "u_dev"), (f_dev, "f_dev"), (r_dev, "r_dev")):
         _check_field(t, n)
         _check_shape(t, tuple(u_host.shape), n)
-    flags = SAFARA_FLAG_STRICT if strict else 0
+    flags = (SAFARA_FLAG_STRICT if strict else 0) | (SAFARA_FLAG_PIPELINE if pipeline else 0)
     check(lib().safara_rhs_host(u_host.data_ptr(), f_host.data_ptr(), r_host.data_ptr(),
                                 u_dev.data_ptr(), f_dev.data_ptr(), r_dev.data_ptr(),
                                 nx, ny, nz, ctypes.byref(coeffs), flags, int(nchunks),
@@ -291,7 +293,8 @@ def rhs_host(u_host: torch.Tensor, f_host: torch.Tensor, r_host: torch.Tensor,
 
 def rhs_host_ex(u_host: torch.Tensor, f_host: torch.Tensor, r_host: torch.Tensor,
                 u_dev: torch.Tensor, f_dev: torch.Tensor, r_dev: torch.Tensor, dims: Dims,
-                coeffs: Coeffs, strict: bool = False, nchunks: int = 8, stream=None):
+                coeffs: Coeffs, strict: bool = False, nchunks: int = 8, stream=None,
+                pipeline: bool = False):
     """End-to-end pass on host (pinned) arrays in the layout `dims` describes
     (e.g. the unpadded sy = nx layout) through device buffers of the same layout."""
     need = (_max_offset(dims, dims.nz) + 1)
@@ -304,7 +307,7 @@ def rhs_host_ex(u_host: torch.Tensor, f_host: torch.Tensor, r_host: torch.Tensor
         _check_field(t, n)
         if t.numel() < need:
             raise ValueError(f"{n}: {t.numel()} elements < the descriptor's {need}")
-    flags = SAFARA_FLAG_STRICT if strict else 0
+    flags = (SAFARA_FLAG_STRICT if strict else 0) | (SAFARA_FLAG_PIPELINE if pipeline else 0)
     check(lib().safara_rhs_host_ex(u_host.data_ptr(), f_host.data_ptr(), r_host.data_ptr(),
                                    u_dev.data_ptr(), f_dev.data_ptr(), r_dev.data_ptr(),
                                    ctypes.byref(dims), ctypes.byref(coeffs), flags, int(nchunks),

@@ -341,3 +341,25 @@ def test_host_e2e_unpadded_descriptor(cls, nchunks):
     torch.cuda.synchronize()
     got = hr.permute(0, 2, 3, 1).numpy()
     assert np.array_equal(got, oracle_rhs(inp))
+
+
+@pytest.mark.parametrize("cls,nchunks", [(("SP", "W"), 3), (("BT", "C"), 8)])
+def test_host_e2e_pipelined_calls(cls, nchunks):
+    """SAFARA_FLAG_PIPELINE: four back-to-back host calls on DIFFERENT inputs
+    through the same device buffers, no synchronisation in between (the next
+    call's H2D overlaps this call's last kernels and D2H): every call's rhs is
+    still bit-identical (STRICT) to the oracle on its own inputs."""
+    n = 4
+    inps = [nasgen.make_class(*cls, seed=20 + s) for s in range(n)]
+    nz, ny, nx, _ = inps[0].u.shape
+    hus = [sr.pack(i.u, pin=True) for i in inps]
+    hfs = [sr.pack(i.forcing, pin=True) for i in inps]
+    hrs = [torch.zeros_like(hus[0]).pin_memory() for _ in range(n)]
+    du, df, dr = (torch.empty(hus[0].shape, dtype=torch.float64, device="cuda") for _ in range(3))
+    c = sr.coeffs_nas(nx, ny, nz, inps[0].dt)
+    for s in range(n):
+        sr.rhs_host(hus[s], hfs[s], hrs[s], du, df, dr, nx, c, strict=True, nchunks=nchunks,
+                    pipeline=True)
+    torch.cuda.synchronize()
+    for s in range(n):
+        assert np.array_equal(sr.unpack(hrs[s], nx), oracle_rhs(inps[s])), f"call {s}"
