@@ -41,7 +41,7 @@ def parse():
     ap.add_argument("--strict", action="store_true", help="time the STRICT variant")
     ap.add_argument("--dist", action="store_true",
                     help="use the z-slab/NCCL path even on one rank (testing)")
-    ap.add_argument("--e2e-steps", type=int, default=5)
+    ap.add_argument("--e2e-steps", type=int, default=20)
     ap.add_argument("--e2e-chunks", type=int, default=8,
                     help="k-chunks of the pipelined H2D / compute / D2H e2e path")
     ap.add_argument("--workload", default="rhs", choices=["rhs", "rhs_aux", "rhs_norm", "rhs_aux_norm", "seismic_dz",
