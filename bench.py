@@ -433,14 +433,30 @@ def run_single(args):
     ev = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps + 1)]
     l0 = sr.launch_count()
     torch.cuda.synchronize()
+    # window events (stream launches only): 5 equal windows of the K passes,
+    # for the min / median per-pass spread SURVEY §8(d) asks about
+    nwin = 5 if (graph is None and not args.launch_events and args.steps >= 10) else 0
+    wev = {args.steps * w // nwin: torch.cuda.Event(enable_timing=True)
+           for w in range(1, nwin)} if nwin else {}
     ev[0].record(stream)
     for k in range(replays if graph is not None else args.steps):
         step()
         if args.launch_events and graph is None:
             ev[k + 1].record(stream)
+        elif k + 1 in wev:
+            wev[k + 1].record(stream)
     if not args.launch_events or graph is not None:
         ev[-1].record(stream)
     torch.cuda.synchronize()
+    windows = None
+    if nwin:
+        bounds = [0] + sorted(wev) + [args.steps]
+        evs = [ev[0]] + [wev[b] for b in sorted(wev)] + [ev[-1]]
+        wms = sorted(evs[w].elapsed_time(evs[w + 1]) * 1e3 / (bounds[w + 1] - bounds[w])
+                     for w in range(nwin))
+        windows = {"n": nwin, "us_per_pass_min": round(wms[0], 2),
+                   "us_per_pass_median": round(wms[nwin // 2], 2),
+                   "us_per_pass_max": round(wms[-1], 2)}
     launches = sr.launch_count() - l0 + (per_graph_launches * replays if graph is not None else 0)
     total_ms = ev[0].elapsed_time(ev[-1])
     # one launch per step: the average launch duration is the step time
@@ -515,6 +531,7 @@ def run_single(args):
                    "launch": (f"CUDA graph of {args.graph} passes, replayed {replays}x"
                               if graph is not None else "one stream launch per pass")},
         "hbm_gbs": achieved,
+        "windows": windows,
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "peak_kind": peak_kind, "traffic": traffic,
                      "bytes_per_point": bytes_per_point, "kernel_ms": kern_ms,

@@ -40,6 +40,10 @@ def run(args):
         os.environ.setdefault("MASTER_PORT", "29511")
     if same_gpu:
         local = 0
+        if args.halo == "nccl" and world > 1:
+            # NCCL itself refuses two ranks of one communicator on one device
+            raise SystemExit("SAFARA_SAME_GPU=1 supports only --halo peer: NCCL does not allow "
+                             "two ranks on one GPU (the NCCL halo needs one GPU per rank)")
     torch.cuda.set_device(local)
     if same_gpu:
         dist.init_process_group("gloo", rank=rank, world_size=world)
