@@ -51,6 +51,9 @@ __device__ __forceinline__ void ws_pwait(uint64_t *bar, uint32_t parity) {
 #ifndef SAFARA_WS_NORM_PROBE
 #define SAFARA_WS_NORM_PROBE 0  // timing probe: the fused norm without its in-loop accumulation (wrong norm)
 #endif
+#ifndef SAFARA_WS_LATE_FULL
+#define SAFARA_WS_LATE_FULL 0  // 1: wait for plane k+2's tile just before its own-column read
+#endif
 #ifndef SAFARA_WS_CSLEEP
 #define SAFARA_WS_CSLEEP 0      // consumer waits: suspend-time hint (ns), 0 = plain try_wait spin
 #endif
@@ -293,7 +296,9 @@ __device__ __forceinline__ void ws_step(SegW &g, const Params &P, int k, int q, 
     // this step
     if (!FAST) {
         ws_cwait(&ws_afull()[(q + 1) % WS_US], (uint32_t)((q + 1) / WS_US) & 1u);
+#if !SAFARA_WS_LATE_FULL
         ws_cwait(&ws_full()[(q + 2) % WS_US], (uint32_t)((q + 2) / WS_US) & 1u);
+#endif
     }
     const double *const s2 = su + (size_t)((q + 2) % WS_US) * U_SLOT;
     double an[5];
@@ -397,6 +402,12 @@ __device__ __forceinline__ void ws_step(SegW &g, const Params &P, int k, int q, 
     }
 #if !SAFARA_ZETA_FIRST
     zeta();
+#endif
+#if SAFARA_WS_LATE_FULL
+    // plane k+2's tile is read only here (own column): wait for it here, so
+    // the first step of a pass computes plane k's xi/eta/zeta while plane
+    // k+2 is still arriving (the ring-fill latency of short slab passes)
+    if (!FAST) ws_cwait(&ws_full()[(q + 2) % WS_US], (uint32_t)((q + 2) / WS_US) & 1u);
 #endif
     if (PEER && !FAST && k + 2 >= P.pk_hi)
         peer_col(an, P, k + 2, g.colo);  // f2: the upper neighbour's own column
