@@ -52,7 +52,7 @@ __device__ __forceinline__ void ws_pwait(uint64_t *bar, uint32_t parity) {
 #define SAFARA_WS_NORM_PROBE 0  // timing probe: the fused norm without its in-loop accumulation (wrong norm)
 #endif
 #ifndef SAFARA_WS_LATE_FULL
-#define SAFARA_WS_LATE_FULL 0  // 1: wait for plane k+2's tile just before its own-column read
+#define SAFARA_WS_LATE_FULL 1  // wait for plane k+2's tile just before its own-column read (A/B: -0.6 %, profiles/ab_late_placement_r02s2.txt)
 #endif
 #ifndef SAFARA_WS_CSLEEP
 #define SAFARA_WS_CSLEEP 0      // consumer waits: suspend-time hint (ns), 0 = plain try_wait spin
