@@ -54,6 +54,9 @@ __device__ __forceinline__ void ws_pwait(uint64_t *bar, uint32_t parity) {
 #ifndef SAFARA_WS_LATE_FULL
 #define SAFARA_WS_LATE_FULL 1  // wait for plane k+2's tile just before its own-column read (A/B: -0.6 %, profiles/ab_late_placement_r02s2.txt)
 #endif
+#ifndef SAFARA_WS_FORCING_LAST
+#define SAFARA_WS_FORCING_LAST 0  // production: add forcing at the end of the step
+#endif
 #ifndef SAFARA_WS_CSLEEP
 #define SAFARA_WS_CSLEEP 0      // consumer waits: suspend-time hint (ns), 0 = plain try_wait spin
 #endif
@@ -276,26 +279,34 @@ __device__ __forceinline__ void ws_step(SegW &g, const Params &P, int k, int q, 
         ws_cwait(&ws_afull()[(q + 1) % WS_US], (uint32_t)((q + 1) / WS_US) & 1u);
         ws_cwait(&ws_full()[(q + 2) % WS_US], (uint32_t)((q + 2) / WS_US) & 1u);
     }
-    {   // forcing(k): its own ring, released right after this read
+    // forcing(k): its own ring, released right after this read.  FLAST
+    // (production, zeta first): the step starts from the zeta partial sum and
+    // adds forcing at its end, so the forcing wait leaves the top of the step
+    // (the sum of the formed terms re-associated: reading c6)
+    constexpr bool FLAST = SAFARA_WS_FORCING_LAST && SAFARA_ZETA_FIRST && !SAFARA_STRICT_BUILD &&
+                           !FAST;
+    auto read_forcing = [&](double (&f)[5]) {
         if (!FAST) ws_cwait(&ws_ffull()[q % WS_FS], (uint32_t)(q / WS_FS) & 1u);
         const double *fs = ws_f() + (size_t)(q % WS_FS) * F_SLOT;
-#pragma unroll
         // own forcing: (ty, tx+1) of the FX-wide tile = aux-tile index - AXW
         static_assert(FX == AXW, "forcing and aux tiles share the row width");
-        for (int m = 0; m < 5; ++m) acc[m] = fs[m * TY * FX - AXW + g.ac];
+#pragma unroll
+        for (int m = 0; m < 5; ++m) f[m] = fs[m * TY * FX - AXW + g.ac];
         if (g.fidx >= 0) {  // one i-face value of this row: rhs = forcing (reading c3)
             __stcs(g.fptr, fs[g.fidx]);
             g.fptr += SK(r);
         }
         __syncwarp();
         if ((threadIdx.x & 31) == 0) mbar_arrive(&ws_fempty()[q % WS_FS]);
-    }
+    };
+    if (!FLAST) read_forcing(acc);
     // the aux of plane k+1 (own rho_i / square for the zeta flux) is in place
     // and plane k+2's tile has landed (own column read at the end of the
     // step); plane k+2's aux is not needed yet, so its evaluation overlaps
     // this step
     if (!FAST) {
-        ws_cwait(&ws_afull()[(q + 1) % WS_US], (uint32_t)((q + 1) / WS_US) & 1u);
+        // zeta last: the aux of plane k+1 is first needed by zeta (below)
+        if (SAFARA_ZETA_FIRST) ws_cwait(&ws_afull()[(q + 1) % WS_US], (uint32_t)((q + 1) / WS_US) & 1u);
 #if !SAFARA_WS_LATE_FULL
         ws_cwait(&ws_full()[(q + 2) % WS_US], (uint32_t)((q + 2) / WS_US) & 1u);
 #endif
@@ -330,7 +341,7 @@ __device__ __forceinline__ void ws_step(SegW &g, const Params &P, int k, int q, 
             p.rho = o1.x; p.sq = o1.y;
         }
         qn.rho = g.rq; qn.sq = g.sq;
-        flux_dir<3, false, UD>(acc, wz, vc, qsc, pc, p, qn, C, 2);
+        flux_dir<3, FLAST, UD>(acc, wz, vc, qsc, pc, p, qn, C, 2);
     };
 #if SAFARA_ZETA_FIRST
     zeta();
@@ -401,6 +412,7 @@ __device__ __forceinline__ void ws_step(SegW &g, const Params &P, int k, int q, 
         diss_apply(acc, t, C.dssp);
     }
 #if !SAFARA_ZETA_FIRST
+    if (!FAST) ws_cwait(&ws_afull()[(q + 1) % WS_US], (uint32_t)((q + 1) / WS_US) & 1u);
     zeta();
 #endif
 #if SAFARA_WS_LATE_FULL
@@ -431,6 +443,12 @@ __device__ __forceinline__ void ws_step(SegW &g, const Params &P, int k, int q, 
         diss_apply(acc, t_z, C.dssp);
     }
 #endif
+    if (FLAST) {
+        double fv[5];
+        read_forcing(fv);
+#pragma unroll
+        for (int m = 0; m < 5; ++m) acc[m] = acc[m] + fv[m];
+    }
     if (FAST) {  // predicated stores: no branch
         double *rp = g.rptr;
 #pragma unroll
